@@ -1,0 +1,460 @@
+"""Pins of the CPU oracle against things other than itself (-m "not gpu").
+
+Each test names what fixes the expected value: a published constant, a hand-worked example,
+a closed form, an independent library routine (numpy / torch conversions), or brute force.
+"""
+import itertools
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+import torch
+
+from oracle import pyoracle as po
+
+L = po.lib()
+PHI = 0x9E3779B97F4A7C15
+
+
+def golden(golden_dir, name):
+    with open(os.path.join(golden_dir, name)) as f:
+        return json.load(f)
+
+
+# --------------------------------------------------------------------------- hashing (App. A)
+
+def test_mix_is_published_splitmix64(golden_dir):
+    """mix = SplitMix64 finaliser: key(0, i) = mix(i*phi) is the i-th SplitMix64 output from
+    state 0, whose first values are published with the reference implementation."""
+    g = golden(golden_dir, "appendix_a.json")
+    got = [L.or_key(0, i) for i in range(1, 5)]
+    assert got == [int(x, 16) for x in g["splitmix64_seed0_first4"]]
+
+
+def test_appendix_a_golden_vectors(golden_dir):
+    """SURVEY App. A golden vectors (independent Python rendering of the spec, seed 42)."""
+    g = golden(golden_dir, "appendix_a.json")
+    s = g["seed"]
+    S = L.or_stream(s, 1, 0, 0)
+    assert S == int(g["S_SHUF"], 16)
+    assert [L.or_key(S, i) for i in range(3)] == [int(x, 16) for x in g["key_S_SHUF_0_2"]]
+    assert po.perm(S, 10).tolist() == g["perm_S_SHUF_10"]
+    pr = po.perm(L.or_stream(s, 2, 0, 0), 10)
+    assert pr.tolist() == g["perm_S_ROW_10"]
+    assert po.perm(L.or_stream(s, 6, 0, 0), 8).tolist() == g["perm_S_HW_0_0_8"]
+    for i, want in enumerate(g["perm_S_WF_0_0_i_8"]):
+        assert po.perm(L.or_stream(s, 7, 0, i), 8).tolist() == want
+    assert po.perm(L.or_stream(s, 8, 0, 0), 8).tolist() == g["pi_0_a8"]
+    # the same values through a whole oracle context (relabel, strata order, init)
+    m = 10
+    o = po.Oracle(m, 10, 16, [0], [0], [1.0], seed=s, grid_a=8)
+    assert o.export("rho_r").tolist() == g["rho_R_10"]
+    assert o.export("strata", 0).tolist() == g["pi_0_a8"]
+    P, _ = o.factors()
+    np.testing.assert_allclose(P[0, :4], g["init_k16_P0_0_3_fp32"], rtol=2e-7)
+    o16 = po.Oracle(m, 10, 16, [0], [0], [1.0], seed=s, storage="fp16")
+    P16, _ = o16.factors()
+    np.testing.assert_allclose(P16[0, :4], g["init_k16_P0_0_3_fp16"], rtol=5e-4)
+
+
+def test_keys_distinct_and_perm_is_sorted_permutation():
+    S = L.or_stream(7, 1, 0, 0)
+    n = 200_000
+    p = po.perm(S, n)
+    assert np.array_equal(np.sort(p), np.arange(n))
+    keys = np.array([L.or_key(S, int(i)) for i in p[:2000]], dtype=np.uint64)
+    assert np.all(keys[1:] > keys[:-1])
+
+
+# --------------------------------------------------------------------------- storage rounding
+
+def _probe_floats(n=400_000, seed=0):
+    rng = np.random.default_rng(seed)
+    mant = rng.integers(0, 1 << 23, n, dtype=np.uint32)
+    expo = rng.integers(127 - 30, 127 + 17, n, dtype=np.uint32)  # spans subnormal..overflow
+    sign = rng.integers(0, 2, n, dtype=np.uint32) << 31
+    x = (sign | (expo << 23) | mant).view(np.float32)
+    # exact halfway cases of fp16 normals and subnormals, and the overflow boundary
+    half_ties = (np.arange(1, 2000, dtype=np.float32) + 0.5) * np.float32(2.0 ** -24)
+    extra = np.array([0.0, -0.0, 65504.0, 65519.99, 65520.0, 2.0 ** -25, 2.0 ** -25 * 1.0000001,
+                      2.0 ** -24, 6.1035156e-05, 1.0 + 2.0 ** -11, 1.0 + 3 * 2.0 ** -11],
+                     dtype=np.float32)
+    return np.concatenate([x, half_ties, -half_ties, extra])
+
+
+def test_f16_encoder_matches_numpy_ieee_rne():
+    """The oracle's software binary16 encoder vs numpy's IEEE round-to-nearest-even cast."""
+    x = _probe_floats()
+    with np.errstate(over="ignore"):
+        want = x.astype(np.float16).view(np.uint16)
+    got = np.array([L.or_f16_bits(float(v)) for v in x], dtype=np.uint16)
+    bad = np.nonzero(got != want)[0]
+    assert bad.size == 0, (x[bad[:5]], got[bad[:5]], want[bad[:5]])
+    back = np.array([L.or_f16_value(int(h)) for h in want[:20000]], dtype=np.float32)
+    np.testing.assert_array_equal(back, want[:20000].view(np.float16).astype(np.float32))
+
+
+def test_bf16_encoder_matches_torch_rne():
+    x = _probe_floats(200_000, seed=1)
+    x = x[np.abs(x) < 1e30]
+    want = torch.from_numpy(x).to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16)
+    got = np.array([L.or_bf16_bits(float(v)) for v in x], dtype=np.uint16)
+    assert np.array_equal(got, want)
+
+
+# --------------------------------------------------------------------------- one update
+
+def test_hand_update_dyadic_exact(golden_dir):
+    """Alg. 1 l.8-10 by hand (dyadic: exact in fp32 and fp16)."""
+    h = golden(golden_dir, "hand_update.json")["dyadic"]
+    for storage in ("fp32", "fp16", "bf16"):
+        p, q = po.update(h["p"], h["q"], h["r"], h["gamma"], h["lambda"], h["lambda"], storage)
+        assert p.tolist() == h["p_new"]
+        assert q.tolist() == h["q_new"]
+        assert q.tolist() != h["q_new_if_sequential_reading"]
+
+
+def test_hand_update_nondyadic(golden_dir):
+    h = golden(golden_dir, "hand_update.json")["nondyadic"]
+    p, q = po.update(h["p"], h["q"], h["r"], h["gamma"], h["lambda"], h["lambda"])
+    np.testing.assert_allclose(p, h["p_new"], atol=h["tol"])
+    np.testing.assert_allclose(q, h["q_new"], atol=h["tol"])
+
+
+def test_update_is_half_gradient_step_of_eq3():
+    """Central finite differences of Eq. 3 equal 2(p - p')/gamma (R2): the update is a
+    gradient step with gamma absorbing the factor 2.  Fails for a dropped term, a wrong sign,
+    a swapped p/q, or the sequential reading of line 10."""
+    rng = np.random.default_rng(3)
+    for trial in range(20):
+        k = int(rng.choice([1, 2, 7, 16]))
+        p = rng.normal(size=k).astype(np.float32)
+        q = rng.normal(size=k).astype(np.float32)
+        r = float(rng.normal() * 2)
+        lp, lq = float(rng.uniform(0, 1)), float(rng.uniform(0, 1))
+        g = 0.05
+        p1, q1 = po.update(p, q, r, g, lp, lq)
+        h = 1e-6
+        gp = np.zeros(k)
+        gq = np.zeros(k)
+        pd, qd = p.astype(np.float64), q.astype(np.float64)
+        for d in range(k):
+            e = np.zeros(k); e[d] = h
+            gp[d] = (po.sample_loss(pd + e, qd, r, lp, lq) - po.sample_loss(pd - e, qd, r, lp, lq)) / (2 * h)
+            gq[d] = (po.sample_loss(pd, qd + e, r, lp, lq) - po.sample_loss(pd, qd - e, r, lp, lq)) / (2 * h)
+        step_p = 2 * (pd - p1.astype(np.float64)) / g
+        step_q = 2 * (qd - q1.astype(np.float64)) / g
+        np.testing.assert_allclose(step_p, gp, rtol=2e-3, atol=2e-3)
+        np.testing.assert_allclose(step_q, gq, rtol=2e-3, atol=2e-3)
+
+
+def test_update_special_cases():
+    rng = np.random.default_rng(4)
+    p = rng.normal(size=16).astype(np.float32)
+    q = rng.normal(size=16).astype(np.float32)
+    # gamma = 0: nothing moves
+    p1, q1 = po.update(p, q, 3.0, 0.0, 0.3, 0.3)
+    assert np.array_equal(p1, p) and np.array_equal(q1, q)
+    # lambda = 0 and r = p.q exactly: fixed point (dyadic values so the dot is exact)
+    pe = np.array([0.5, -1.25, 2.0], dtype=np.float32)
+    qe = np.array([1.5, 0.25, -0.75], dtype=np.float32)
+    r = float(np.dot(pe.astype(np.float64), qe))
+    p1, q1 = po.update(pe, qe, r, 0.1, 0.0, 0.0)
+    assert np.array_equal(p1, pe) and np.array_equal(q1, qe)
+    # k = 1, lambda = 0: e' = e (1 - g (p^2 + q^2) - g^2 e p q)   (closed form, in double)
+    pp, qq, rr, g = 0.7, -0.4, 1.3, 0.05
+    e = rr - pp * qq
+    p1, q1 = po.update([pp], [qq], rr, g, 0.0, 0.0)
+    e_new = rr - float(p1[0]) * float(q1[0])
+    assert abs(e_new - e * (1 - g * (pp * pp + qq * qq) - g * g * e * pp * qq)) < 1e-6
+    # ... and repeating it converges p.q -> r geometrically
+    P, Q = np.float32([pp]), np.float32([qq])
+    for _ in range(400):
+        P, Q = po.update(P, Q, rr, g, 0.0, 0.0)
+    assert abs(rr - float(P[0]) * float(Q[0])) < 1e-5
+
+
+def test_gamma_schedule_closed_form():
+    """Eq. 9 at t = 0 (gamma_0 = alpha, R4) and at perfect squares, where t^1.5 is an
+    integer; plus Table 3 Netflix values (alpha .08, beta .3)."""
+    for a, b in [(0.08, 0.3), (0.08, 0.2), (0.05, 0.0), (1.0, 1.0)]:
+        a32, b32 = float(np.float32(a)), float(np.float32(b))
+        assert L.or_gamma(a, b, 0) == np.float32(a)
+        for t, t15 in [(1, 1), (4, 8), (9, 27), (16, 64), (100, 1000)]:
+            assert L.or_gamma(a, b, t) == np.float32(a32 / (1 + b32 * t15))
+    want = [0.08, 0.06153846, 0.043277673, 0.031264096]
+    got = [L.or_gamma(0.08, 0.3, t) for t in range(4)]
+    np.testing.assert_allclose(got, want, rtol=1e-7)
+    assert all(x > y for x, y in zip(got, got[1:]))
+
+
+# --------------------------------------------------------------------------- schedules
+
+def _tiny_uniform(m=60, n=50, N=3000, seed=5):
+    rng = np.random.default_rng(seed)
+    return (rng.integers(0, m, N).astype(np.int32), rng.integers(0, n, N).astype(np.int32),
+            rng.normal(size=N).astype(np.float32), m, n)
+
+
+SCHEDULES = [
+    dict(schedule="hogwild", batch_f=7),
+    dict(schedule="hogwild", batch_f=256),
+    dict(schedule="wavefront", workers=4, wf_cols=8),
+    dict(schedule="wavefront", workers=3, wf_cols=5),
+    dict(schedule="wavefront", workers=4, wf_cols=8, cyclic=True),
+    dict(schedule="hogwild", batch_f=16, grid_a=8),
+    dict(schedule="wavefront", workers=2, wf_cols=3, grid_a=4),
+]
+
+
+@pytest.mark.parametrize("kw", SCHEDULES)
+def test_every_sample_exactly_once_per_epoch(kw):
+    u, v, r, m, n = _tiny_uniform()
+    o = po.Oracle(m, n, 4, u, v, r, **kw)
+    for t in range(3):
+        order = o.export("order", t)
+        assert np.array_equal(np.sort(order), np.arange(len(u)))
+
+
+def test_serial_special_cases_reduce_to_algorithm_1():
+    """s = c = a = 1 wavefront and f >= N Hogwild both run the storage order verbatim
+    (Alg. 1: one shuffled pass)."""
+    u, v, r, m, n = _tiny_uniform()
+    for kw in (dict(schedule="wavefront", workers=1, wf_cols=1),
+               dict(schedule="hogwild", batch_f=1 << 20)):
+        o = po.Oracle(m, n, 4, u, v, r, **kw)
+        assert np.array_equal(o.export("order", 0), np.arange(len(u)))
+    # and training in that order equals the update applied by hand in storage order
+    o = po.Oracle(m, n, 4, u, v, r, schedule="wavefront", workers=1, wf_cols=1, seed=9)
+    P, Q = o.factors()
+    perm = o.export("perm")
+    g = L.or_gamma(0.08, 0.3, 0)
+    for i in perm:
+        P[u[i]], Q[v[i]] = po.update(P[u[i]], Q[v[i]], float(r[i]), g, 0.05, 0.05)
+    o.train_epoch()
+    P2, Q2 = o.factors()
+    assert np.array_equal(P, P2) and np.array_equal(Q, Q2)
+
+
+def test_hogwild_chunks_are_consecutive_storage_runs():
+    u, v, r, m, n = _tiny_uniform()
+    f = 64
+    o = po.Oracle(m, n, 4, u, v, r, schedule="hogwild", batch_f=f)
+    order = o.export("order", 1)
+    co = o.export("chunkorder", 1)
+    assert np.array_equal(np.sort(co), np.arange(len(co)))
+    want = np.concatenate([np.arange(c * f, min((c + 1) * f, len(u))) for c in co])
+    assert np.array_equal(order, want)
+    # a permutation of chunks that changes with the epoch
+    assert not np.array_equal(co, o.export("chunkorder", 0))
+
+
+def test_wavefront_tickets_brute_force_and_fig6_golden(golden_dir):
+    """Ticket rank of (w,i) = #earlier visits (lexicographic (w,i)) of the same column.
+    Golden: seed 42, s=4, c=8: workers 0, 1, 3 all start at column 0 -> tickets 0, 1, 2
+    (the Fig. 6 narrative P:L287-289 of a worker waiting for a column)."""
+    g = golden(golden_dir, "appendix_a.json")
+    s, c = 4, 8
+    o = po.Oracle(20, 20, 2, [0], [0], [1.0], seed=42, schedule="wavefront", workers=s, wf_cols=c)
+    seq = o.export("wfseq", 0).reshape(s, c)
+    assert seq.tolist() == g["perm_S_WF_0_0_i_8"]
+    tk = o.export("tickets", 0).reshape(s, c)
+    assert [tk[0, 0], tk[1, 0], tk[3, 0]] == [0, 1, 2]
+    for i in range(s):
+        for w in range(c):
+            col = seq[i, w]
+            cnt = sum(1 for w2 in range(c) for i2 in range(s)
+                      if (w2, i2) < (w, i) and seq[i2, w2] == col)
+            assert tk[i, w] == cnt
+    # every column is visited exactly s times per epoch: ranks 0..s-1 per column
+    for col in range(c):
+        assert sorted(tk[seq == col].tolist()) == list(range(s))
+
+
+def test_wavefront_cyclic_has_no_same_wave_column_conflicts():
+    s, c = 5, 9
+    o = po.Oracle(30, 30, 2, [0], [0], [1.0], schedule="wavefront", workers=s, wf_cols=c,
+                  cyclic=True)
+    seq = o.export("wfseq", 3).reshape(s, c)
+    for i in range(s):
+        assert sorted(seq[i].tolist()) == list(range(c))
+    for w in range(c):
+        assert len(set(seq[:, w].tolist())) == s
+
+
+def test_wavefront_blocks_respect_eq6_within_a_wave_order():
+    """Replaying the oracle's order, two updates of the same row sub-block or column sub-block
+    never interleave across different blocks: each (i,j) block runs contiguously, and a
+    worker's blocks appear in its wave order."""
+    u, v, r, m, n = _tiny_uniform(N=4000)
+    s, c = 4, 8
+    o = po.Oracle(m, n, 4, u, v, r, schedule="wavefront", workers=s, wf_cols=c)
+    blk = o.export("blockid", 0)
+    order = o.export("order", 0)
+    seq = o.export("wfseq", 0).reshape(s, c)
+    runs = [blk[order[0]]]
+    for j in order[1:]:
+        if blk[j] != runs[-1]:
+            runs.append(blk[j])
+    assert len(runs) == len(set(runs))          # each block is one contiguous run
+    pos = {b: x for x, b in enumerate(runs)}
+    for i in range(s):
+        ids = [i * c + seq[i, w] for w in range(c) if (i * c + seq[i, w]) in pos]
+        assert [pos[b] for b in ids] == sorted(pos[b] for b in ids)
+
+
+def test_block_assignment_segments_are_balanced_and_consistent():
+    u, v, r, m, n = _tiny_uniform(m=97, n=61, N=5000)
+    a = 8
+    o = po.Oracle(m, n, 4, u, v, r, grid_a=a)
+    rho_r, rho_c = o.export("rho_r"), o.export("rho_c")
+    assert np.array_equal(np.sort(rho_r), np.arange(m))
+    assert np.array_equal(np.sort(rho_c), np.arange(n))
+    seg_r = rho_r * a // m
+    sizes = np.bincount(seg_r, minlength=a)
+    assert sizes.max() - sizes.min() <= 1
+    blk = o.export("blockid")
+    perm = o.export("perm")
+    assert np.array_equal(blk, seg_r[u[perm]] * a + (rho_c[v[perm]] * a // n))
+
+
+def _feasible_orders_2x2():
+    """Fig. 15: 2x2 blocks, 2 workers; an order b1 b2 b3 b4 is feasible iff the
+    concurrently running pairs (b1,b2) and (b3,b4) are independent (Eq. 6 at block level)."""
+    rc = {1: (0, 0), 2: (0, 1), 3: (1, 0), 4: (1, 1)}
+
+    def indep(x, y):
+        return rc[x][0] != rc[y][0] and rc[x][1] != rc[y][1]
+
+    return [o for o in itertools.permutations([1, 2, 3, 4]) if indep(o[0], o[1]) and indep(o[2], o[3])]
+
+
+def test_fig15_feasible_block_orders_and_strata_order():
+    feas = _feasible_orders_2x2()
+    assert len(feas) == 8 and len(list(itertools.permutations(range(4)))) == 24
+    # the strata order with a = 2 run by 2 workers is always one of the feasible orders,
+    # and every stratum's a blocks are pairwise independent for a = 8
+    u, v, r, m, n = _tiny_uniform()
+    o2 = po.Oracle(m, n, 2, u, v, r, grid_a=2)
+    for t in range(6):
+        pi = o2.export("strata", t)
+        order = tuple(1 + rr * 2 + (rr + pi[j]) % 2 for j in range(2) for rr in range(2))
+        assert order in feas
+    o8 = po.Oracle(m, n, 2, u, v, r, grid_a=8)
+    for t in range(3):
+        pi = o8.export("strata", t)
+        assert sorted(pi.tolist()) == list(range(8))
+        for j in range(8):
+            cols = [(rr + pi[j]) % 8 for rr in range(8)]
+            assert len(set(cols)) == 8
+
+
+def test_run_block_in_strata_order_equals_train_epoch():
+    u, v, r, m, n = _tiny_uniform()
+    kw = dict(schedule="wavefront", workers=2, wf_cols=3, grid_a=4, seed=11)
+    a = 4
+    o1 = po.Oracle(m, n, 4, u, v, r, **kw)
+    o2 = po.Oracle(m, n, 4, u, v, r, **kw)
+    for t in range(2):
+        o1.train_epoch()
+        pi = o2.export("strata", t)
+        for j in range(a):
+            for rr in range(a):
+                o2.run_block(t, rr * a + (rr + pi[j]) % a)
+    o2.set_epoch(2)
+    assert np.array_equal(o1.factors()[0], o2.factors()[0])
+    assert np.array_equal(o1.factors()[1], o2.factors()[1])
+
+
+# --------------------------------------------------------------------------- training
+
+def _tiny_set():
+    from paper_conf_hpdc_xietfl17_b200 import synth
+    return synth.tiny(seed=0)
+
+
+def test_init_distribution():
+    """Alg. 1 l.3: U[0, a), a = sqrt(1/(k*scale)) (R5)."""
+    k = 16
+    o = po.Oracle(1000, 800, k, [0], [0], [0.0], init_scale=1.0)
+    P, Q = o.factors()
+    a = math.sqrt(1 / k)
+    for X in (P, Q):
+        assert X.min() >= 0 and X.max() < a
+        assert abs(X.mean() - a / 2) < 0.01 * a
+    o2 = po.Oracle(1000, 800, k, [0], [0], [0.0], init_scale=4.0)
+    assert o2.factors()[0].max() < math.sqrt(1 / (4 * k))
+
+
+def test_rmse_textbook_and_closed_forms():
+    R = _tiny_set()
+    o = po.Oracle(R.m, R.n, 16, R.u, R.v, R.r)
+    o.train_epoch()
+    P, Q = o.factors()
+    pred = np.einsum("ij,ij->i", P[R.ut].astype(np.float64), Q[R.vt].astype(np.float64))
+    want = np.sqrt(np.mean((R.rt.astype(np.float64) - pred) ** 2))
+    assert abs(o.rmse(R.ut, R.vt, R.rt) - want) < 1e-5 * want
+    # P = 0: prediction 0, RMSE = sqrt(mean r^2); rating_scale multiplies back
+    o.set_factors(P=np.zeros_like(P))
+    assert abs(o.rmse(R.ut, R.vt, R.rt) - np.sqrt(np.mean(R.rt.astype(np.float64) ** 2))) < 1e-6
+    o4 = po.Oracle(R.m, R.n, 16, R.u, R.v, R.r, rating_scale=4.0)
+    o4.set_factors(P=np.zeros_like(P))
+    assert abs(o4.rmse(R.ut, R.vt, R.rt) - np.sqrt(np.mean(R.rt.astype(np.float64) ** 2))) < 1e-5
+
+
+def test_loss_is_eq2_sum():
+    R = _tiny_set()
+    o = po.Oracle(R.m, R.n, 16, R.u[:500], R.v[:500], R.r[:500], lambda_p=0.1, lambda_q=0.2)
+    P, Q = o.factors()
+    p, q = P[R.u[:500]].astype(np.float64), Q[R.v[:500]].astype(np.float64)
+    e = R.r[:500].astype(np.float64) - (p * q).sum(1)
+    lp, lq = float(np.float32(0.1)), float(np.float32(0.2))  # the oracle holds lambda as float
+    want = (e ** 2 + lp * (p ** 2).sum(1) + lq * (q ** 2).sum(1)).sum()
+    assert abs(o.loss() - want) < 1e-9 * want
+
+
+@pytest.mark.parametrize("schedule", ["hogwild", "wavefront"])
+def test_training_loss_monotone_table3_netflix(schedule):
+    """Eq. 2 decreases every epoch on tiny with Table 3 Netflix parameters."""
+    R = _tiny_set()
+    kw = dict(workers=8, wf_cols=16) if schedule == "wavefront" else {}
+    o = po.Oracle(R.m, R.n, 16, R.u, R.v, R.r, lambda_p=0.05, alpha=0.08, beta=0.3,
+                  schedule=schedule, **kw)
+    losses = [o.loss()]
+    for _ in range(10):
+        o.train_epoch()
+        losses.append(o.loss())
+    assert all(b < a for a, b in zip(losses, losses[1:])), losses
+
+
+def test_planted_recovery():
+    """Planted rank-4 noiseless tiny set: SGD recovers it (SURVEY 8(c) calibration)."""
+    R = _tiny_set()
+    std = float(np.std(R.r))
+    o = po.Oracle(R.m, R.n, 16, R.u, R.v, R.r, lambda_p=0.05, alpha=0.08, beta=0.3)
+    for _ in range(10):
+        o.train_epoch()
+    assert o.rmse(R.ut, R.vt, R.rt) <= 0.30 * std
+    o = po.Oracle(R.m, R.n, 16, R.u, R.v, R.r, lambda_p=0.0, alpha=0.05, beta=0.0)
+    for _ in range(40):
+        o.train_epoch()
+    assert o.rmse(R.ut, R.vt, R.rt) <= 0.10 * std
+    assert o.rmse(R.u, R.v, R.r) <= 0.03 * std
+
+
+def test_fp16_storage_keeps_values_representable():
+    R = _tiny_set()
+    o = po.Oracle(R.m, R.n, 16, R.u, R.v, R.r, storage="fp16")
+    o.train_epoch()
+    P, Q = o.factors()
+    for X in (P, Q):
+        assert np.array_equal(X.astype(np.float16).astype(np.float32), X)
+
+
+def test_create_rejects_bad_input():
+    with pytest.raises(ValueError):
+        po.Oracle(10, 10, 4, [10], [0], [1.0])
+    with pytest.raises(ValueError):
+        po.Oracle(10, 10, 4, [0], [0], [float("nan")])
