@@ -1,0 +1,183 @@
+/*
+ * include/mf.h -- C ABI of libmf_b200.so, the B200-native hot path of cuMF_SGD
+ * (Xie, Tan, Fong, Liang, "CuMF_SGD: Parallelized Stochastic Gradient Descent for Matrix
+ * Factorization on GPUs", HPDC'17).  "P:L<n>" cites a line of the paper text
+ * (/root/reference/PAPER.md), "A:" the index/RNG specification of SURVEY.md Appendix A, and
+ * "R<n>" a reading of a silent or garbled passage listed in DESIGN.md section 3.
+ *
+ * Problem (Eq. 1-3): R (m x n, N observed ratings r_{u,v}) ~ P (m x k) x Q (k x n).
+ * Per rating, Algorithm 1 lines 8-10:
+ *     e = r - p_u . q_v ;  p_u += gamma_t (e q_v - lambda_p p_u) ;  q_v += gamma_t (e p_u - lambda_q q_v)
+ * (both from the pre-update p_u, q_v -- R1), gamma_t = alpha / (1 + beta t^1.5)  (Eq. 9),
+ * scheduled by batch-Hogwild! (section 5.1) or by the deterministic wavefront
+ * (section 5.2) inside DSGD-style strata across GPUs (section 6.1).
+ *
+ * Conventions (all entry points):
+ *  - Every call returns mf_status (0 = MF_OK, < 0 = error); nothing throws or aborts across the
+ *    ABI.  mf_last_error(ctx) returns a NUL-terminated message for the last error of a ctx.
+ *  - A CUDA error is sticky: the call returns MF_E_CUDA and every later call on that ctx
+ *    returns MF_E_STATE.  NCCL errors likewise (MF_E_NCCL).
+ *  - Ownership: the caller owns every buffer it passes in or receives results into (host or
+ *    device, see each on_device flag); the ctx owns all of its device state, allocated through
+ *    params.alloc when given (else cudaMallocAsync on the ctx stream), freed by mf_destroy.
+ *  - One ctx per device (per rank); a ctx is not thread-safe.
+ *  - Call order: mf_create -> mf_load_coo(MF_TRAIN) [-> mf_load_coo(MF_TEST)] ->
+ *    { mf_train_epoch | mf_rmse | mf_get_factors | mf_set_factors | mf_export_schedule }*
+ *    -> mf_destroy.  Out of order, or a second load of the same set, returns MF_E_STATE.
+ *  - Work is enqueued on params.stream (a cudaStream_t, e.g. torch.cuda.current_stream()),
+ *    or on a ctx-created stream when NULL.  mf_train_epoch does not synchronise; mf_rmse,
+ *    mf_get_factors, mf_export_schedule and mf_get_stats do.
+ *  - Index types: N is int64 (Hugewiki-shaped N = 3.07e9 > 2^31); u, v are int32.
+ */
+#ifndef MF_B200_H
+#define MF_B200_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MF_ABI_VERSION 1
+
+typedef struct mf_ctx mf_ctx; /* opaque, owned by the library */
+
+typedef int32_t mf_status;
+enum {
+  MF_OK = 0,
+  MF_E_INVAL = -1,       /* bad argument / parameter                                  */
+  MF_E_NOMEM = -2,       /* device or host allocation failed                          */
+  MF_E_CUDA = -3,        /* CUDA runtime error (sticky)                               */
+  MF_E_NCCL = -4,        /* NCCL error or NCCL unavailable for world > 1 (sticky)     */
+  MF_E_STATE = -5,       /* call out of order, or ctx already in an error state        */
+  MF_E_RANGE = -6,       /* rating index out of [0,m)x[0,n), non-finite r, NaN RMSE    */
+  MF_E_UNSUPPORTED = -7  /* k not in {16,32,64,128,256}, too many workers, no device  */
+};
+
+typedef enum { MF_FP32 = 0, MF_FP16 = 1, MF_BF16 = 2 } mf_storage;   /* P:L242 feature storage */
+typedef enum { MF_HOGWILD = 0, MF_WAVEFRONT = 1 } mf_schedule;      /* section 5.1 / 5.2 */
+typedef enum { MF_TRAIN = 0, MF_TEST = 1 } mf_set;
+
+/* Device-memory hooks (e.g. torch's caching allocator).  alloc returns NULL on failure. */
+typedef struct mf_allocator {
+  void* (*alloc)(size_t bytes, void* stream, void* user);
+  void (*free)(void* ptr, size_t bytes, void* stream, void* user);
+  void* user;
+} mf_allocator;
+
+typedef struct mf_params {
+  uint32_t struct_size;   /* = sizeof(mf_params) (ABI check)                                   */
+  int64_t m, n;           /* R is m x n                                                */
+  int32_t k;              /* feature dimension (Table 2 k = 128); {16,32,64,128,256}     */
+  float lambda_p;         /* Eq. 2 regularisers; the paper uses one lambda (R3)          */
+  float lambda_q;
+  float alpha, beta;      /* Eq. 9 learning-rate schedule (Table 3)                 */
+  float init_scale;       /* Alg. 1 l.3 scale_factor: P,Q ~ U[0, sqrt(1/(k*init_scale))) (R5)    */
+  float rating_scale;     /* r' = r / rating_scale for training; RMSE reported x rating_scale   */
+  uint64_t seed;          /* keys every random choice (A: streams S_SHUF ... S_ST)              */
+  int32_t schedule;       /* mf_schedule                                                        */
+  int32_t storage;        /* mf_storage of P and Q; arithmetic is always fp32                   */
+  int32_t workers;        /* s: Hogwild = concurrent sample groups (0 = all resident);
+                             wavefront = row sub-blocks per strata block (0 = 2048)             */
+  int32_t batch_f;        /* Eq. 8 batch f (0 = 256)                                    */
+  int32_t wf_cols;        /* wavefront column sub-blocks c (0 = 2*s, R9)                        */
+  int32_t grid_a;         /* strata grid a x a (0 = 1 if world == 1 else 8); a % world == 0      */
+  int32_t cyclic;         /* wavefront: 1 = cyclic column order (A: cyclic variant), needs c >= s */
+  int32_t lane_bytes;     /* Hogwild/RMSE kernel: bytes of p_u (and q_v) per lane, 16 or 32 (0 = 16) */
+  int32_t device;         /* CUDA device ordinal                                                */
+  int32_t rank, world;    /* world > 1: DSGD strata over `world` GPUs, one ctx per rank         */
+  int32_t transport;      /* 0 = NCCL (world > 1)                                              */
+  const void* nccl_id;    /* 128-byte ncclUniqueId, identical on all ranks (world > 1)          */
+  void* stream;           /* cudaStream_t or NULL                                               */
+  const mf_allocator* alloc; /* NULL = cudaMallocAsync                                          */
+} mf_params;
+
+/* Fill *p with defaults (Table 3 Netflix lambda/alpha/beta, k = 128, fp32, Hogwild, f = 256). */
+mf_status mf_params_default(mf_params* p);
+
+/* Validate parameters, select the device, create/adopt the stream; world > 1 also initialises
+ * the NCCL communicator from nccl_id (libnccl.so.2 is dlopen'ed; missing -> MF_E_NCCL).
+ * Returns MF_E_INVAL / MF_E_UNSUPPORTED for bad params; *out is NULL on error. */
+mf_status mf_create(const mf_params* p, mf_ctx** out);
+
+/* Load a rating set in COO form: nnz triples (u[i], v[i], r[i]) (2 ints + 1 float),
+ * host or device pointers (on_device = 0/1); the library copies them and never keeps the
+ * caller's pointers.  MF_TRAIN runs the one-time preprocessing on the GPU:
+ *   validation (MF_E_RANGE if u or v out of range or r non-finite; the ctx stays usable),
+ *   Alg. 1 l.2 random_shuffle (storage order = perm(S_SHUF, nnz), A),
+ *   row/column relabel (A: S_ROW, S_COL) and bucketing into strata blocks / wavefront
+ *   sub-blocks, Alg. 1 l.3 initialisation of P, Q (A: S_P, S_Q).
+ * world > 1: every rank passes the FULL set; a rank keeps only the blocks it owns.
+ * MF_TEST stores the test set (relabelled, scaled) for mf_rmse. */
+mf_status mf_load_coo(mf_ctx* ctx, int32_t set, int64_t nnz, const int32_t* u, const int32_t* v,
+                      const float* r, int32_t on_device);
+
+/* Enqueue one epoch t (t = ctx epoch counter, 0-based, R4) on the stream: gamma_t (Eq. 9),
+ * the epoch schedule (chunk order / column sequences / tickets, A) and the SGD kernels; for
+ * world > 1 the a sub-epochs each followed by the NCCL Q-segment rotation.  Increments t and
+ * writes it to *epoch_done when non-NULL.  Does not synchronise. */
+mf_status mf_train_epoch(mf_ctx* ctx, int32_t* epoch_done);
+
+/* RMSE of the chosen set (R13): rating_scale * sqrt(sum (r' - p_u.q_v)^2 / N), fp32 dots,
+ * fp64 accumulation, deterministic reduction order.  world > 1: global value (all ranks).
+ * Synchronises.  MF_E_RANGE if the result is NaN (divergence). */
+mf_status mf_rmse(mf_ctx* ctx, int32_t set, double* out);
+
+/* Copy the model out in ORIGINAL ids as fp32 (Alg. 1 l.15 model_shuffle): P is m x k
+ * row-major, Q is n x k row-major (row v = q_v, R14).  Either pointer may be NULL.
+ * world > 1: gathers all segments; every rank receives the full P and Q.  Synchronises. */
+mf_status mf_get_factors(mf_ctx* ctx, float* P, float* Q, int32_t on_device);
+
+/* Overwrite P and/or Q (same layout as mf_get_factors), rounded to the storage type (RNE). */
+mf_status mf_set_factors(mf_ctx* ctx, const float* P, const float* Q, int32_t on_device);
+
+/* Set / get the epoch counter t (checkpoint-resume). */
+mf_status mf_set_epoch(mf_ctx* ctx, int32_t t);
+mf_status mf_get_epoch(const mf_ctx* ctx, int32_t* t);
+
+/* Export an index structure for bit-exact comparison (tests).  Host int64 buffer; with
+ * buf == NULL only *len is set to the required element count; otherwise *len must be >= it.
+ * Layouts are identical to the oracle's exports. */
+enum {
+  MF_EX_PERM = 0,       /* [N]  caller index of storage position j                     */
+  MF_EX_RHO_R = 1,      /* [m]  row relabel rank                                       */
+  MF_EX_RHO_C = 2,      /* [n]  column relabel rank                                    */
+  MF_EX_BLOCKID = 3,    /* [N]  per storage position: block b (Hogwild) or
+                                b*(s*c) + i*c + j (wavefront)                           */
+  MF_EX_CHUNKORDER = 4, /* [sum_b nchunks_b] Hogwild chunk order per block, b ascending (epoch) */
+  MF_EX_WFSEQ = 5,      /* [a*a*s*c] seq_i[w] per block b, worker i, wave w (epoch)     */
+  MF_EX_TICKETS = 6,    /* [a*a*s*c] ticket rank of visit (w,i), stored [b][i][w] (epoch) */
+  MF_EX_STRATA = 7      /* [a]  pi_t (epoch)                                            */
+};
+mf_status mf_export_schedule(mf_ctx* ctx, int32_t what, int32_t epoch, int64_t* buf, int64_t* len);
+
+/* Timing of the last mf_train_epoch, from CUDA events recorded on the ctx stream around the
+ * work (synchronises).  sgd_ms: SGD kernel launches only; sched_ms: schedule build;
+ * comm_ms: Q rotation; launches: kernels launched by the epoch. */
+typedef struct mf_stats {
+  double epoch_ms, sgd_ms, sched_ms, comm_ms;
+  int64_t sgd_launches, launches;
+  int64_t updates;          /* samples updated by this rank in the epoch */
+  int64_t bytes_per_update; /* algorithmic: 12 + 4*k*sizeof(storage) (north_star; Eq. 5)  */
+  int32_t workers, lanes, grid, block;
+} mf_stats;
+mf_status mf_get_stats(mf_ctx* ctx, mf_stats* out);
+
+/* Host-only strata planner (no GPU needed): which rank trains block row-segment r in
+ * sub-epoch j of epoch t, and which Q segments move before sub-epoch j.  For each segment
+ * J in [0,a): holder[J] = rank that holds (trains with) segment J during sub-epoch j.
+ * A: the stratum of sub-epoch j is {(r, (r + pi_t[j]) mod a)}; rank g owns row segments
+ * [g*a/G, (g+1)*a/G).  Returns MF_E_INVAL if a % world != 0. */
+mf_status mf_strata_holders(uint64_t seed, int32_t a, int32_t world, int32_t t, int32_t j,
+                            int32_t* holder);
+
+void mf_destroy(mf_ctx* ctx);
+const char* mf_last_error(const mf_ctx* ctx);
+const char* mf_status_string(mf_status s);
+int32_t mf_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MF_B200_H */

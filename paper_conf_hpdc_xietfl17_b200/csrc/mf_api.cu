@@ -1,0 +1,1388 @@
+// mf_api.cu -- host runtime of libmf_b200.so: the C ABI of include/mf.h, the one-time GPU
+// preprocessing (validate, shuffle, relabel, bucket, init), the per-epoch schedule build
+// (chunk order, column sequences, tickets) and the epoch driver.  All device work runs in
+// this library's kernels (plus CUB radix sort as the sort primitive); nothing falls back to
+// the CPU.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <cub/cub.cuh>
+#include <string>
+#include <vector>
+
+#include "mf.h"
+#include "mf_comm.h"
+#include "mf_internal.h"
+
+using namespace mfb;
+
+// =============================================================================================
+// preprocessing / schedule kernels
+// =============================================================================================
+namespace {
+
+__global__ void k_validate(const int32_t* __restrict__ u, const int32_t* __restrict__ v,
+                           const float* __restrict__ r, int64_t N, int64_t m, int64_t n,
+                           int* __restrict__ bad) {
+  int local = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t a = u[i], b = v[i];
+    const float x = r[i];
+    if (a < 0 || a >= m || b < 0 || b >= n || !isfinite(x)) local = 1;
+  }
+  if (__syncthreads_or(local) && threadIdx.x == 0) atomicOr(bad, 1);
+}
+
+// keys[i] = key(S, i), vals[i] = i  (A: "perm(S, n) = [0..n) sorted ascending by key(S,.)")
+__global__ void k_iota_keys(uint64_t S, int64_t n, uint64_t* __restrict__ keys,
+                            uint32_t* __restrict__ vals) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    keys[i] = hkey(S, (uint64_t)i);
+    vals[i] = (uint32_t)i;
+  }
+}
+
+// rho[perm[j]] = j
+__global__ void k_rank_of(const uint32_t* __restrict__ perm, int64_t n, int32_t* __restrict__ rho) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n;
+       j += (int64_t)gridDim.x * blockDim.x)
+    rho[perm[j]] = (int32_t)j;
+}
+
+struct Grid {
+  int64_t m, n, a, s, c;  // s, c only for wavefront
+  bool wf;
+};
+
+__device__ __forceinline__ int64_t seg_lo(int64_t r, int64_t a, int64_t n) {
+  return cdiv64(r * n, a);
+}
+
+// Bucket of a (relabelled) sample: strata block b = r*a + J, and for the wavefront the
+// sub-block (b*s + i)*c + j inside it (A: "Segments and blocks").
+__device__ __forceinline__ uint32_t bucket_of(const Grid& G, int64_t ru, int64_t rc) {
+  const int64_t r = ru * G.a / G.m, J = rc * G.a / G.n;
+  const int64_t b = r * G.a + J;
+  if (!G.wf) return (uint32_t)b;
+  const int64_t rlo = seg_lo(r, G.a, G.m), rhi = seg_lo(r + 1, G.a, G.m);
+  const int64_t clo = seg_lo(J, G.a, G.n), chi = seg_lo(J + 1, G.a, G.n);
+  const int64_t i = (ru - rlo) * G.s / (rhi - rlo);
+  const int64_t j = (rc - clo) * G.c / (chi - clo);
+  return (uint32_t)((b * G.s + i) * G.c + j);
+}
+
+// storage order j (Alg. 1 l.2): sample perm[j], relabelled and scaled; plus its bucket.
+__global__ void k_build_storage(const uint32_t* __restrict__ perm, int64_t N,
+                                const int32_t* __restrict__ u, const int32_t* __restrict__ v,
+                                const float* __restrict__ r, const int32_t* __restrict__ rho_r,
+                                const int32_t* __restrict__ rho_c, double rs, Grid G,
+                                Rating* __restrict__ stor, uint32_t* __restrict__ bucket,
+                                uint32_t* __restrict__ pos) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < N;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t i = perm[j];
+    Rating x;
+    x.u = rho_r[u[i]];
+    x.v = rho_c[v[i]];
+    x.r = (float)((double)r[i] / rs);     // R5: r' = r / rating_scale, rounded once
+    stor[j] = x;
+    if (bucket) bucket[j] = bucket_of(G, x.u, x.v);
+    if (pos) pos[j] = (uint32_t)j;
+  }
+}
+
+__global__ void k_build_test(const int32_t* __restrict__ u, const int32_t* __restrict__ v,
+                             const float* __restrict__ r, int64_t N,
+                             const int32_t* __restrict__ rho_r, const int32_t* __restrict__ rho_c,
+                             double rs, Rating* __restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    Rating x;
+    x.u = rho_r[u[i]];
+    x.v = rho_c[v[i]];
+    x.r = (float)((double)r[i] / rs);
+    out[i] = x;
+  }
+}
+
+__global__ void k_histogram(const uint32_t* __restrict__ bucket, int64_t N,
+                            unsigned int* __restrict__ cnt) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < N;
+       j += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(cnt + bucket[j], 1u);
+}
+
+// Place sorted sample x (bucket b = key[x]) at slot dst_off[b] + (x - src_off[b]).
+__global__ void k_place(const uint32_t* __restrict__ keys_sorted,
+                        const uint32_t* __restrict__ pos_sorted, int64_t N,
+                        const int64_t* __restrict__ src_off, const int64_t* __restrict__ dst_off,
+                        const Rating* __restrict__ stor, Rating* __restrict__ slots,
+                        uint32_t* __restrict__ slot_pos) {
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < N;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t b = keys_sorted ? keys_sorted[x] : 0u;
+    const uint32_t j = pos_sorted[x];
+    const int64_t slot = dst_off[b] + (x - src_off[b]);
+    slots[slot] = stor[j];
+    if (slot_pos) slot_pos[slot] = j;
+  }
+}
+
+// Alg. 1 l.3 (R5): X[rho[id]][d] = round_S((float)U24(S, id*k+d) * 2^-24 * amp),
+// keyed by the ORIGINAL id (A: S_P / S_Q).
+template <typename T>
+__global__ void k_init(T* __restrict__ X, const int32_t* __restrict__ rho, int64_t rows, int k,
+                       uint64_t S, float amp) {
+  const int64_t total = rows * k;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t id = x / k, d = x % k;
+    const float u01 = (float)(hkey(S, (uint64_t)x) >> 40) * 0x1p-24f;
+    const float val = u01 * amp;
+    X[(int64_t)rho[id] * k + d] = static_cast<T>(val);
+  }
+}
+
+template <typename T> __device__ __forceinline__ float to_f32(T x) { return static_cast<float>(x); }
+template <> __device__ __forceinline__ float to_f32<__half>(__half x) { return __half2float(x); }
+template <> __device__ __forceinline__ float to_f32<__nv_bfloat16>(__nv_bfloat16 x) {
+  return __bfloat162float(x);
+}
+template <typename T> __device__ __forceinline__ T from_f32(float x);
+template <> __device__ __forceinline__ float from_f32<float>(float x) { return x; }
+template <> __device__ __forceinline__ __half from_f32<__half>(float x) { return __float2half_rn(x); }
+template <> __device__ __forceinline__ __nv_bfloat16 from_f32<__nv_bfloat16>(float x) {
+  return __float2bfloat16_rn(x);
+}
+
+// model_shuffle (Alg. 1 l.15): out[id][d] = fp32(X[rho[id]][d])
+template <typename T>
+__global__ void k_unrelabel(const T* __restrict__ X, const int32_t* __restrict__ rho, int64_t rows,
+                            int k, float* __restrict__ out) {
+  const int64_t total = rows * k;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t id = x / k, d = x % k;
+    out[x] = to_f32<T>(X[(int64_t)rho[id] * k + d]);
+  }
+}
+template <typename T>
+__global__ void k_relabel_store(T* __restrict__ X, const int32_t* __restrict__ rho, int64_t rows,
+                                int k, const float* __restrict__ in) {
+  const int64_t total = rows * k;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t id = x / k, d = x % k;
+    X[(int64_t)rho[id] * k + d] = from_f32<T>(in[x]);
+  }
+}
+
+// Hogwild chunk keys of epoch t: global chunk gc of block b (local q = gc - choff[b]) gets
+// key(S_HW(t,b), q) (A).  nb <= 64 blocks -> linear search is fine.
+__global__ void k_chunk_keys(const int64_t* __restrict__ choff, int nb, uint64_t seed, int32_t t,
+                             uint64_t* __restrict__ keys, uint32_t* __restrict__ vals) {
+  const int64_t total = choff[nb];
+  for (int64_t gc = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; gc < total;
+       gc += (int64_t)gridDim.x * blockDim.x) {
+    int b = 0;
+    while (gc >= choff[b + 1]) ++b;
+    const uint64_t S = make_stream(seed, kTagHW, (uint64_t)t, (uint64_t)b);
+    keys[gc] = hkey(S, (uint64_t)(gc - choff[b]));
+    vals[gc] = (uint32_t)gc;
+  }
+}
+
+// block id of each (sorted) chunk, for the stable second pass
+__global__ void k_chunk_block(const uint32_t* __restrict__ vals, const int64_t* __restrict__ choff,
+                              int nb, int64_t total, uint32_t* __restrict__ blk) {
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t gc = vals[x];
+    int b = 0;
+    while (gc >= choff[b + 1]) ++b;
+    blk[x] = (uint32_t)b;
+  }
+}
+
+// wavefront column-sequence keys: item (b*s + i)*c + j gets key(S_WF(t,b,i), j) (A).
+__global__ void k_wf_keys(int64_t nseg, int s, int c, uint64_t seed, int32_t t,
+                          uint64_t* __restrict__ keys, uint32_t* __restrict__ vals) {
+  const int64_t total = nseg * c;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t sg = x / c, j = x % c;
+    const int64_t b = sg / s, i = sg % s;
+    const uint64_t S = make_stream(seed, kTagWF, (uint64_t)t, ((uint64_t)b << 32) + (uint64_t)i);
+    keys[x] = hkey(S, (uint64_t)j);
+    vals[x] = (uint32_t)x;
+  }
+}
+
+// generic: keys for nseg independent permutations of length c with per-segment stream
+// make_stream(seed, tag, t, seg) (cyclic variant's tau / sigma per block)
+__global__ void k_perm_keys(int64_t nseg, int c, uint64_t seed, uint64_t tag, int32_t t,
+                            uint64_t* __restrict__ keys, uint32_t* __restrict__ vals) {
+  const int64_t total = nseg * c;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t sg = x / c, j = x % c;
+    keys[x] = hkey(make_stream(seed, tag, (uint64_t)t, (uint64_t)sg), (uint64_t)j);
+    vals[x] = (uint32_t)x;
+  }
+}
+
+__global__ void k_seg_of(const uint32_t* __restrict__ vals, int64_t total, int c,
+                         uint32_t* __restrict__ seg) {
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x)
+    seg[x] = (uint32_t)(vals[x] / (uint32_t)c);
+}
+
+// sorted (segment-major) vals -> position-in-segment j values
+__global__ void k_mod_c(const uint32_t* __restrict__ vals, int64_t total, int c,
+                        int32_t* __restrict__ out) {
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x)
+    out[x] = (int32_t)(vals[x] % (uint32_t)c);
+}
+
+// cyclic variant (A): seq_i[w] = sigma[(tau[i] + w) mod c] per block b
+__global__ void k_cyclic_seq(const int32_t* __restrict__ tau, const int32_t* __restrict__ sigma,
+                             int64_t nb, int s, int c, int32_t* __restrict__ seq) {
+  const int64_t total = nb * s * (int64_t)c;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t w = x % c, bi = x / c, i = bi % s, b = bi / s;
+    seq[x] = sigma[b * c + (tau[b * c + i] + w) % c];
+  }
+}
+
+// ticket keys: visit (b,i,w) to column col = seq[(b*s+i)*c+w] gets key ((b*c+col)*c + w)*s + i
+__global__ void k_ticket_keys(const int32_t* __restrict__ seq, int64_t nb, int s, int c,
+                              uint64_t* __restrict__ keys, uint32_t* __restrict__ vals) {
+  const int64_t total = nb * s * (int64_t)c;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t w = x % c, bi = x / c, i = bi % s, b = bi / s;
+    const int64_t col = seq[x];
+    keys[x] = (uint64_t)(((b * c + col) * c + w) * s + i);
+    vals[x] = (uint32_t)x;
+  }
+}
+
+// rank of visit = sorted position - first position of its (b, col) group (each column is
+// visited exactly s times per block and epoch).
+__global__ void k_ticket_rank(const uint32_t* __restrict__ vals, int64_t total, int s,
+                              int32_t* __restrict__ rank) {
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x)
+    rank[vals[x]] = (int32_t)(x % s);
+}
+
+int bits_for(uint64_t maxval) {
+  int b = 1;
+  while (b < 64 && (maxval >> b) != 0) ++b;
+  return b;
+}
+
+inline int grid_for(int64_t n, int num_sms) {
+  int64_t b = (n + 255) / 256;
+  int64_t cap = (int64_t)num_sms * 16;
+  if (b > cap) b = cap;
+  if (b < 1) b = 1;
+  return (int)b;
+}
+
+// Eq. 9, t 0-based (R4): evaluated in double with t^1.5 = t*sqrt(t), rounded once.
+float gamma_of(float alpha, float beta, int32_t t) {
+  const double td = (double)t;
+  return (float)((double)alpha / (1.0 + (double)beta * td * std::sqrt(td)));
+}
+
+// A: host perm of a small set (strata order pi_t).
+std::vector<int64_t> host_perm(uint64_t S, int64_t n) {
+  std::vector<std::pair<uint64_t, int64_t>> t((size_t)n);
+  for (int64_t i = 0; i < n; ++i) t[(size_t)i] = {hkey(S, (uint64_t)i), i};
+  std::sort(t.begin(), t.end());
+  std::vector<int64_t> out((size_t)n);
+  for (int64_t i = 0; i < n; ++i) out[(size_t)i] = t[(size_t)i].second;
+  return out;
+}
+
+}  // namespace
+
+// =============================================================================================
+// context
+// =============================================================================================
+struct mf_ctx {
+  mf_params p{};
+  uint8_t nccl_id[128]{};
+  int dev = 0, num_sms = 0;
+  cudaStream_t st = nullptr;
+  bool own_stream = false;
+  mf_status sticky = MF_OK;
+  std::string err;
+  bool train_loaded = false, test_loaded = false;
+
+  int64_t m = 0, n = 0, N = 0, Ntest = 0;
+  int k = 0, a = 1, s = 1, c = 1, f = 256, G = 1, rank = 0;
+  int32_t t = 0;
+  bool wf = false;
+
+  // device state
+  Rating* slots = nullptr;         int64_t nslots = 0;
+  uint32_t* slot_pos = nullptr;    // storage position of each slot (0xFFFFFFFF = pad)
+  uint32_t* perm = nullptr;        // caller index of storage position j
+  int32_t* rho_r = nullptr;
+  int32_t* rho_c = nullptr;
+  void* P = nullptr;
+  void* Q = nullptr;
+  Rating* test = nullptr;
+  int64_t* sub_off = nullptr;      // wavefront: a*a*s*c + 1
+  std::vector<int64_t> blk_off;    // a*a + 1 slot offsets (Hogwild: padded to f)
+  std::vector<int64_t> blk_len;    // a*a sample counts
+  std::vector<int64_t> ch_off;     // a*a + 1 chunk offsets (Hogwild)
+  int64_t* d_choff = nullptr;
+  // schedule scratch
+  uint64_t *sk0 = nullptr, *sk1 = nullptr;
+  uint32_t *sv0 = nullptr, *sv1 = nullptr, *sb = nullptr;
+  int64_t sched_cap = 0;
+  uint32_t* chunk_order = nullptr;  // Hogwild: sorted global chunk ids, blocks ascending
+  int32_t *seq = nullptr, *rank_arr = nullptr, *tickets = nullptr;
+  int32_t *tau = nullptr, *sigma = nullptr;
+  unsigned long long* counter = nullptr;
+  double* rm_partial = nullptr;
+  double* rm_out = nullptr;
+  void* tmp = nullptr;
+  size_t tmp_bytes = 0;
+  int sched_built_for = -1;
+
+  // stats
+  std::vector<cudaEvent_t> ev;     // pairs for SGD launches
+  cudaEvent_t ev_e0 = nullptr, ev_e1 = nullptr, ev_s0 = nullptr, ev_s1 = nullptr;
+  cudaEvent_t ev_c0 = nullptr, ev_c1 = nullptr;
+  int n_sgd = 0, n_launch = 0;
+  int64_t updates = 0;
+  int last_workers = 0, last_lanes = 0, last_grid = 0, last_block = 0;
+  bool have_stats = false;
+  std::vector<double> comm_ms_acc;
+
+  mf::Comm* comm = nullptr;
+
+  mf_status fail(mf_status s, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    err = buf;
+    if (s == MF_E_CUDA || s == MF_E_NCCL) sticky = s;
+    return s;
+  }
+  mf_status cuda_fail(cudaError_t e, const char* what, int line) {
+    cudaGetLastError();
+    if (e == cudaErrorMemoryAllocation) return fail(MF_E_NOMEM, "%s: out of device memory (line %d)", what, line);
+    return fail(MF_E_CUDA, "%s: %s (line %d)", what, cudaGetErrorString(e), line);
+  }
+  mf_status enter() {
+    if (sticky != MF_OK) return fail(MF_E_STATE, "ctx is in an error state after: %s", err.c_str());
+    cudaError_t e = cudaSetDevice(dev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaSetDevice", __LINE__);
+    return MF_OK;
+  }
+
+  template <typename X>
+  mf_status alloc(X** out, size_t count) {
+    *out = nullptr;
+    size_t bytes = count * sizeof(X);
+    if (bytes == 0) bytes = 16;
+    void* ptr = nullptr;
+    if (p.alloc && p.alloc->alloc) {
+      ptr = p.alloc->alloc(bytes, (void*)st, p.alloc->user);
+      if (!ptr) return fail(MF_E_NOMEM, "allocator returned NULL for %zu bytes", bytes);
+    } else {
+      cudaError_t e = cudaMallocAsync(&ptr, bytes, st);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(MF_E_NOMEM, "cudaMallocAsync(%zu): %s", bytes, cudaGetErrorString(e));
+      }
+    }
+    sizes.push_back({ptr, bytes});
+    *out = static_cast<X*>(ptr);
+    return MF_OK;
+  }
+  template <typename X>
+  void release(X*& ptr) {
+    if (!ptr) return;
+    size_t bytes = 0;
+    for (size_t i = 0; i < sizes.size(); ++i)
+      if (sizes[i].first == (void*)ptr) {
+        bytes = sizes[i].second;
+        sizes.erase(sizes.begin() + (long)i);
+        break;
+      }
+    if (p.alloc && p.alloc->free) p.alloc->free((void*)ptr, bytes, (void*)st, p.alloc->user);
+    else cudaFreeAsync((void*)ptr, st);
+    ptr = nullptr;
+  }
+  std::vector<std::pair<void*, size_t>> sizes;
+
+  mf_status need_tmp(size_t bytes) {
+    if (bytes <= tmp_bytes) return MF_OK;
+    release(tmp);
+    tmp_bytes = 0;
+    mf_status s2 = alloc((char**)&tmp, bytes);
+    if (s2) return s2;
+    tmp_bytes = bytes;
+    return MF_OK;
+  }
+  template <typename K, typename V>
+  mf_status sort_pairs(const K* kin, K* kout, const V* vin, V* vout, int64_t n_items, int end_bit) {
+    size_t bytes = 0;
+    cudaError_t e = cub::DeviceRadixSort::SortPairs(nullptr, bytes, kin, kout, vin, vout, n_items, 0,
+                                                    end_bit, st);
+    if (e != cudaSuccess) return cuda_fail(e, "cub sort (size)", __LINE__);
+    mf_status s2 = need_tmp(bytes);
+    if (s2) return s2;
+    e = cub::DeviceRadixSort::SortPairs(tmp, bytes, kin, kout, vin, vout, n_items, 0, end_bit, st);
+    if (e != cudaSuccess) return cuda_fail(e, "cub sort", __LINE__);
+    return MF_OK;
+  }
+  int ssize() const { return p.storage == MF_FP32 ? 4 : 2; }
+  int lo_row_seg() const { return rank * (a / G); }
+  int hi_row_seg() const { return (rank + 1) * (a / G); }
+};
+
+#define TRY(expr)                         \
+  do {                                    \
+    mf_status _s = (expr);                \
+    if (_s != MF_OK) return _s;           \
+  } while (0)
+#define CUDA_TRY(ctx, expr)                                                  \
+  do {                                                                       \
+    cudaError_t _e = (expr);                                                 \
+    if (_e != cudaSuccess) return (ctx)->cuda_fail(_e, #expr, __LINE__);     \
+  } while (0)
+#define KERNEL_TRY(ctx) CUDA_TRY(ctx, cudaGetLastError())
+
+// =============================================================================================
+// C ABI
+// =============================================================================================
+// Definitions take C linkage from the extern "C" declarations in mf.h.
+int32_t mf_abi_version(void) { return MF_ABI_VERSION; }
+
+const char* mf_status_string(mf_status s) {
+  switch (s) {
+    case MF_OK: return "MF_OK";
+    case MF_E_INVAL: return "MF_E_INVAL";
+    case MF_E_NOMEM: return "MF_E_NOMEM";
+    case MF_E_CUDA: return "MF_E_CUDA";
+    case MF_E_NCCL: return "MF_E_NCCL";
+    case MF_E_STATE: return "MF_E_STATE";
+    case MF_E_RANGE: return "MF_E_RANGE";
+    case MF_E_UNSUPPORTED: return "MF_E_UNSUPPORTED";
+  }
+  return "MF_E_?";
+}
+
+const char* mf_last_error(const mf_ctx* ctx) { return ctx ? ctx->err.c_str() : "null ctx"; }
+
+mf_status mf_params_default(mf_params* p) {
+  if (!p) return MF_E_INVAL;
+  std::memset(p, 0, sizeof *p);
+  p->struct_size = (uint32_t)sizeof(mf_params);
+  p->k = 128;
+  p->lambda_p = p->lambda_q = 0.05f;  // Table 3 Netflix
+  p->alpha = 0.08f;
+  p->beta = 0.3f;
+  p->init_scale = 1.0f;
+  p->rating_scale = 1.0f;
+  p->seed = 42;
+  p->schedule = MF_HOGWILD;
+  p->storage = MF_FP32;
+  p->batch_f = 256;
+  p->world = 1;
+  return MF_OK;
+}
+
+mf_status mf_strata_holders(uint64_t seed, int32_t a, int32_t world, int32_t t, int32_t j,
+                            int32_t* holder) {
+  if (a < 1 || world < 1 || a % world != 0 || j < 0 || j >= a || t < 0 || !holder)
+    return MF_E_INVAL;
+  std::vector<int64_t> pi = host_perm(make_stream(seed, kTagStrata, (uint64_t)t, 0), a);
+  const int per = a / world;
+  // segment J is trained in sub-epoch j by the owner of row segment (J - pi_t[j]) mod a
+  for (int J = 0; J < a; ++J) {
+    const int r = (int)(((J - pi[(size_t)j]) % a + a) % a);
+    holder[J] = r / per;
+  }
+  return MF_OK;
+}
+
+mf_status mf_create(const mf_params* p, mf_ctx** out) {
+  if (!out) return MF_E_INVAL;
+  *out = nullptr;
+  if (!p || p->struct_size != sizeof(mf_params)) return MF_E_INVAL;
+  if (p->m <= 0 || p->n <= 0 || p->m >= INT32_MAX || p->n >= INT32_MAX) return MF_E_INVAL;
+  if (!(p->k == 16 || p->k == 32 || p->k == 64 || p->k == 128 || p->k == 256))
+    return MF_E_UNSUPPORTED;
+  if (p->storage < 0 || p->storage > 2 || p->schedule < 0 || p->schedule > 1) return MF_E_INVAL;
+  if (!(p->alpha >= 0.f) || !(p->beta >= 0.f) || !(p->lambda_p >= 0.f) || !(p->lambda_q >= 0.f))
+    return MF_E_INVAL;
+  if (!(p->rating_scale > 0.f) || !(p->init_scale > 0.f)) return MF_E_INVAL;
+  if (p->lane_bytes != 0 && p->lane_bytes != 16 && p->lane_bytes != 32) return MF_E_INVAL;
+  const int world = p->world > 0 ? p->world : 1;
+  if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
+  const int a = p->grid_a > 0 ? p->grid_a : (world == 1 ? 1 : 8);
+  if (a % world != 0 || a > p->m || a > p->n || a > 64) return MF_E_INVAL;
+  if (p->batch_f < 0 || p->workers < 0 || p->wf_cols < 0) return MF_E_INVAL;
+
+  mf_ctx* c = new (std::nothrow) mf_ctx();
+  if (!c) return MF_E_NOMEM;
+  c->p = *p;
+  c->dev = p->device;
+  c->m = p->m;
+  c->n = p->n;
+  c->k = p->k;
+  c->a = a;
+  c->G = world;
+  c->rank = p->rank;
+  c->f = p->batch_f > 0 ? p->batch_f : 256;
+  c->wf = p->schedule == MF_WAVEFRONT;
+  if (c->wf) {
+    const int64_t rows_per_seg = p->m / a;
+    int64_t s = p->workers > 0 ? p->workers : std::min<int64_t>(2048, std::max<int64_t>(1, rows_per_seg / 4));
+    c->s = (int)s;
+    c->c = p->wf_cols > 0 ? p->wf_cols : 2 * c->s;
+    if (p->cyclic && c->c < c->s) { delete c; return MF_E_INVAL; }
+    if ((int64_t)a * a * c->s * c->c >= ((int64_t)1 << 31)) { delete c; return MF_E_UNSUPPORTED; }
+  }
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    delete c;
+    return MF_E_UNSUPPORTED;
+  }
+  if (c->dev < 0 || c->dev >= ndev) { delete c; return MF_E_INVAL; }
+  if (cudaSetDevice(c->dev) != cudaSuccess ||
+      cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, c->dev) != cudaSuccess) {
+    cudaGetLastError();
+    delete c;
+    return MF_E_CUDA;
+  }
+  if (p->stream) {
+    c->st = (cudaStream_t)p->stream;
+  } else {
+    if (cudaStreamCreateWithFlags(&c->st, cudaStreamDefault) != cudaSuccess) {
+      delete c;
+      return MF_E_CUDA;
+    }
+    c->own_stream = true;
+  }
+  cudaEventCreate(&c->ev_e0);
+  cudaEventCreate(&c->ev_e1);
+  cudaEventCreate(&c->ev_s0);
+  cudaEventCreate(&c->ev_s1);
+  cudaEventCreate(&c->ev_c0);
+  cudaEventCreate(&c->ev_c1);
+  if (world > 1) {
+    if (!p->nccl_id) { mf_destroy(c); return MF_E_INVAL; }
+    std::memcpy(c->nccl_id, p->nccl_id, 128);
+    std::string why;
+    c->comm = mf::Comm::create(c->nccl_id, world, p->rank, c->st, &why);
+    if (!c->comm) {
+      c->fail(MF_E_NCCL, "NCCL init failed: %s", why.c_str());
+      mf_destroy(c);
+      return MF_E_NCCL;
+    }
+  }
+  if (c->alloc(&c->counter, 1) || c->alloc(&c->rm_partial, (size_t)c->num_sms * 4) ||
+      c->alloc(&c->rm_out, 2)) {
+    mf_destroy(c);
+    return MF_E_NOMEM;
+  }
+  *out = c;
+  return MF_OK;
+}
+
+void mf_destroy(mf_ctx* c) {
+  if (!c) return;
+  cudaSetDevice(c->dev);
+  if (c->st) cudaStreamSynchronize(c->st);
+  std::vector<std::pair<void*, size_t>> all = c->sizes;
+  for (auto& x : all) {
+    void* ptr = x.first;
+    c->release(ptr);
+  }
+  if (c->st) cudaStreamSynchronize(c->st);
+  for (auto e : c->ev) cudaEventDestroy(e);
+  for (cudaEvent_t e : {c->ev_e0, c->ev_e1, c->ev_s0, c->ev_s1, c->ev_c0, c->ev_c1})
+    if (e) cudaEventDestroy(e);
+  if (c->comm) mf::Comm::destroy(c->comm);
+  if (c->own_stream && c->st) cudaStreamDestroy(c->st);
+  cudaGetLastError();
+  delete c;
+}
+
+// ---------------------------------------------------------------------------------------------
+// load
+// ---------------------------------------------------------------------------------------------
+static mf_status stage_input(mf_ctx* c, int64_t nnz, const int32_t* u, const int32_t* v,
+                             const float* r, int on_device, const int32_t** du,
+                             const int32_t** dv, const float** dr, int32_t** own_u,
+                             int32_t** own_v, float** own_r) {
+  *own_u = nullptr; *own_v = nullptr; *own_r = nullptr;
+  if (on_device) {
+    *du = u; *dv = v; *dr = r;
+    return MF_OK;
+  }
+  TRY(c->alloc(own_u, (size_t)nnz));
+  TRY(c->alloc(own_v, (size_t)nnz));
+  TRY(c->alloc(own_r, (size_t)nnz));
+  CUDA_TRY(c, cudaMemcpyAsync(*own_u, u, nnz * 4, cudaMemcpyHostToDevice, c->st));
+  CUDA_TRY(c, cudaMemcpyAsync(*own_v, v, nnz * 4, cudaMemcpyHostToDevice, c->st));
+  CUDA_TRY(c, cudaMemcpyAsync(*own_r, r, nnz * 4, cudaMemcpyHostToDevice, c->st));
+  *du = *own_u; *dv = *own_v; *dr = *own_r;
+  return MF_OK;
+}
+
+static mf_status validate(mf_ctx* c, int64_t nnz, const int32_t* du, const int32_t* dv,
+                          const float* dr) {
+  int* flag = nullptr;
+  TRY(c->alloc(&flag, 1));
+  CUDA_TRY(c, cudaMemsetAsync(flag, 0, 4, c->st));
+  if (nnz > 0) {
+    k_validate<<<grid_for(nnz, c->num_sms), 256, 0, c->st>>>(du, dv, dr, nnz, c->m, c->n, flag);
+    KERNEL_TRY(c);
+  }
+  int h = 0;
+  CUDA_TRY(c, cudaMemcpyAsync(&h, flag, 4, cudaMemcpyDeviceToHost, c->st));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  c->release(flag);
+  if (h) return c->fail(MF_E_RANGE, "rating index out of range or non-finite rating");
+  return MF_OK;
+}
+
+static mf_status relabel(mf_ctx* c, uint64_t tag, int64_t count, int32_t** rho) {
+  uint64_t *k0 = nullptr, *k1 = nullptr;
+  uint32_t *v0 = nullptr, *v1 = nullptr;
+  TRY(c->alloc(&k0, (size_t)count));
+  TRY(c->alloc(&k1, (size_t)count));
+  TRY(c->alloc(&v0, (size_t)count));
+  TRY(c->alloc(&v1, (size_t)count));
+  TRY(c->alloc(rho, (size_t)count));
+  k_iota_keys<<<grid_for(count, c->num_sms), 256, 0, c->st>>>(make_stream(c->p.seed, tag, 0, 0),
+                                                              count, k0, v0);
+  KERNEL_TRY(c);
+  TRY(c->sort_pairs(k0, k1, v0, v1, count, 64));
+  k_rank_of<<<grid_for(count, c->num_sms), 256, 0, c->st>>>(v1, count, *rho);
+  KERNEL_TRY(c);
+  c->release(k0); c->release(k1); c->release(v0); c->release(v1);
+  return MF_OK;
+}
+
+template <typename T>
+static void launch_init(mf_ctx* c, void* X, const int32_t* rho, int64_t rows, uint64_t S, float amp) {
+  k_init<T><<<grid_for(rows * c->k, c->num_sms), 256, 0, c->st>>>((T*)X, rho, rows, c->k, S, amp);
+}
+
+static mf_status init_factors(mf_ctx* c) {
+  const size_t es = (size_t)c->ssize();
+  TRY(c->alloc((char**)&c->P, (size_t)c->m * c->k * es));
+  TRY(c->alloc((char**)&c->Q, (size_t)c->n * c->k * es));
+  const float amp = (float)std::sqrt(1.0 / ((double)c->k * (double)c->p.init_scale));
+  const uint64_t SP = make_stream(c->p.seed, kTagP, 0, 0), SQ = make_stream(c->p.seed, kTagQ, 0, 0);
+  switch (c->p.storage) {
+    case MF_FP32: launch_init<float>(c, c->P, c->rho_r, c->m, SP, amp);
+                  launch_init<float>(c, c->Q, c->rho_c, c->n, SQ, amp); break;
+    case MF_FP16: launch_init<__half>(c, c->P, c->rho_r, c->m, SP, amp);
+                  launch_init<__half>(c, c->Q, c->rho_c, c->n, SQ, amp); break;
+    default: launch_init<__nv_bfloat16>(c, c->P, c->rho_r, c->m, SP, amp);
+             launch_init<__nv_bfloat16>(c, c->Q, c->rho_c, c->n, SQ, amp); break;
+  }
+  KERNEL_TRY(c);
+  return MF_OK;
+}
+
+static mf_status alloc_schedule(mf_ctx* c) {
+  const int64_t nb = (int64_t)c->a * c->a;
+  int64_t cap = 1;
+  if (c->wf) cap = nb * c->s * (int64_t)c->c;
+  else cap = c->ch_off.back();
+  if (c->wf && c->p.cyclic) cap = std::max<int64_t>(cap, 2 * nb * c->c);
+  cap = std::max<int64_t>(cap, 1);
+  TRY(c->alloc(&c->sk0, (size_t)cap));
+  TRY(c->alloc(&c->sk1, (size_t)cap));
+  TRY(c->alloc(&c->sv0, (size_t)cap));
+  TRY(c->alloc(&c->sv1, (size_t)cap));
+  TRY(c->alloc(&c->sb, (size_t)cap));
+  c->sched_cap = cap;
+  if (c->wf) {
+    TRY(c->alloc(&c->seq, (size_t)cap));
+    TRY(c->alloc(&c->rank_arr, (size_t)cap));
+    TRY(c->alloc(&c->tickets, (size_t)c->c));
+    if (c->p.cyclic) {
+      TRY(c->alloc(&c->tau, (size_t)(nb * c->c)));
+      TRY(c->alloc(&c->sigma, (size_t)(nb * c->c)));
+    }
+  } else {
+    TRY(c->alloc(&c->chunk_order, (size_t)cap));
+  }
+  return MF_OK;
+}
+
+static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_t* v,
+                            const float* r, int on_device) {
+  if (N >= (int64_t)UINT32_MAX) return c->fail(MF_E_UNSUPPORTED, "N >= 2^32 not supported");
+  const int32_t *du, *dv;
+  const float* dr;
+  int32_t *ou, *ov;
+  float* orr;
+  TRY(stage_input(c, N, u, v, r, on_device, &du, &dv, &dr, &ou, &ov, &orr));
+  TRY(validate(c, N, du, dv, dr));
+  c->N = N;
+
+  // Alg. 1 l.2 random_shuffle: storage order = perm(S_SHUF, N)
+  {
+    uint64_t *k0 = nullptr, *k1 = nullptr;
+    uint32_t* v0 = nullptr;
+    TRY(c->alloc(&k0, (size_t)N));
+    TRY(c->alloc(&k1, (size_t)N));
+    TRY(c->alloc(&v0, (size_t)N));
+    TRY(c->alloc(&c->perm, (size_t)N));
+    if (N > 0) {
+      k_iota_keys<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(
+          make_stream(c->p.seed, kTagShuf, 0, 0), N, k0, v0);
+      KERNEL_TRY(c);
+      TRY(c->sort_pairs(k0, k1, v0, c->perm, N, 64));
+    }
+    c->release(k0); c->release(k1); c->release(v0);
+  }
+  // relabel (A: S_ROW, S_COL)
+  TRY(relabel(c, kTagRow, c->m, &c->rho_r));
+  TRY(relabel(c, kTagCol, c->n, &c->rho_c));
+
+  // storage-order samples (relabelled, scaled) and their buckets
+  Grid Gd{c->m, c->n, c->a, c->s, c->c, c->wf};
+  const int64_t nb = (int64_t)c->a * c->a;
+  const int64_t nbuckets = c->wf ? nb * c->s * (int64_t)c->c : nb;
+  Rating* stor = nullptr;
+  uint32_t *bk0 = nullptr, *bk1 = nullptr, *pos0 = nullptr, *pos1 = nullptr;
+  TRY(c->alloc(&stor, (size_t)N));
+  TRY(c->alloc(&bk0, (size_t)N));
+  TRY(c->alloc(&bk1, (size_t)N));
+  TRY(c->alloc(&pos0, (size_t)N));
+  TRY(c->alloc(&pos1, (size_t)N));
+  if (N > 0) {
+    k_build_storage<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(
+        c->perm, N, du, dv, dr, c->rho_r, c->rho_c, (double)c->p.rating_scale, Gd, stor, bk0, pos0);
+    KERNEL_TRY(c);
+  }
+  c->release(ou); c->release(ov); c->release(orr);
+
+  // bucket counts -> offsets
+  unsigned int* cnt = nullptr;
+  TRY(c->alloc(&cnt, (size_t)nbuckets));
+  CUDA_TRY(c, cudaMemsetAsync(cnt, 0, nbuckets * 4, c->st));
+  if (N > 0) {
+    k_histogram<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(bk0, N, cnt);
+    KERNEL_TRY(c);
+  }
+  // stable sort of storage positions by bucket (radix sort is stable; storage order kept, R12)
+  const uint32_t* keys_sorted = nullptr;
+  const uint32_t* pos_sorted = pos0;
+  if (nbuckets > 1 && N > 0) {
+    TRY(c->sort_pairs(bk0, bk1, pos0, pos1, N, bits_for((uint64_t)(nbuckets - 1))));
+    keys_sorted = bk1;
+    pos_sorted = pos1;
+  }
+  int64_t *src_off = nullptr, *dst_off = nullptr;
+  TRY(c->alloc(&src_off, (size_t)nbuckets + 1));
+  if (c->wf) {
+    // sub-block offsets: exclusive scan of the counts (int64)
+    std::vector<unsigned int> hc((size_t)nbuckets);
+    CUDA_TRY(c, cudaMemcpyAsync(hc.data(), cnt, nbuckets * 4, cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    std::vector<int64_t> off((size_t)nbuckets + 1, 0);
+    for (int64_t x = 0; x < nbuckets; ++x) off[(size_t)x + 1] = off[(size_t)x] + hc[(size_t)x];
+    CUDA_TRY(c, cudaMemcpyAsync(src_off, off.data(), (nbuckets + 1) * 8, cudaMemcpyHostToDevice, c->st));
+    c->blk_off.assign((size_t)nb + 1, 0);
+    c->blk_len.assign((size_t)nb, 0);
+    for (int64_t b = 0; b < nb; ++b) {
+      c->blk_off[(size_t)b + 1] = off[(size_t)((b + 1) * c->s * c->c)];
+      c->blk_len[(size_t)b] = c->blk_off[(size_t)b + 1] - c->blk_off[(size_t)b];
+    }
+    c->nslots = N;
+    c->sub_off = src_off;
+    dst_off = src_off;
+    src_off = nullptr;
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));  // host vector `off` goes out of scope
+  } else {
+    // Hogwild: pad every block to a multiple of f (sentinel slots) so chunk q of block b is
+    // slots [blk_off[b] + q f, + f) (A: "Padding").
+    std::vector<unsigned int> hc((size_t)nb);
+    CUDA_TRY(c, cudaMemcpyAsync(hc.data(), cnt, nb * 4, cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    std::vector<int64_t> so((size_t)nb + 1, 0);
+    c->blk_off.assign((size_t)nb + 1, 0);
+    c->blk_len.assign((size_t)nb, 0);
+    c->ch_off.assign((size_t)nb + 1, 0);
+    for (int64_t b = 0; b < nb; ++b) {
+      c->blk_len[(size_t)b] = hc[(size_t)b];
+      so[(size_t)b + 1] = so[(size_t)b] + hc[(size_t)b];
+      const int64_t nch = cdiv64(hc[(size_t)b], c->f);
+      c->ch_off[(size_t)b + 1] = c->ch_off[(size_t)b] + nch;
+      c->blk_off[(size_t)b + 1] = c->blk_off[(size_t)b] + nch * c->f;
+    }
+    c->nslots = c->blk_off.back();
+    TRY(c->alloc(&dst_off, (size_t)nb + 1));
+    CUDA_TRY(c, cudaMemcpyAsync(src_off, so.data(), (nb + 1) * 8, cudaMemcpyHostToDevice, c->st));
+    CUDA_TRY(c, cudaMemcpyAsync(dst_off, c->blk_off.data(), (nb + 1) * 8, cudaMemcpyHostToDevice, c->st));
+    TRY(c->alloc(&c->d_choff, (size_t)nb + 1));
+    CUDA_TRY(c, cudaMemcpyAsync(c->d_choff, c->ch_off.data(), (nb + 1) * 8, cudaMemcpyHostToDevice, c->st));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));  // host vectors used by async copies
+  }
+  TRY(c->alloc(&c->slots, (size_t)std::max<int64_t>(c->nslots, 1)));
+  TRY(c->alloc(&c->slot_pos, (size_t)std::max<int64_t>(c->nslots, 1)));
+  if (c->nslots > N) {
+    CUDA_TRY(c, cudaMemsetAsync(c->slots, 0xFF, c->nslots * sizeof(Rating), c->st));  // u=v=-1
+    CUDA_TRY(c, cudaMemsetAsync(c->slot_pos, 0xFF, c->nslots * 4, c->st));
+  }
+  if (N > 0) {
+    k_place<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(
+        keys_sorted, pos_sorted, N, c->wf ? c->sub_off : src_off, c->wf ? c->sub_off : dst_off,
+        stor, c->slots, c->slot_pos);
+    KERNEL_TRY(c);
+  }
+  if (!c->wf) { c->release(src_off); c->release(dst_off); }
+  c->release(cnt); c->release(stor); c->release(bk0); c->release(bk1);
+  c->release(pos0); c->release(pos1);
+
+  TRY(init_factors(c));
+  TRY(alloc_schedule(c));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  c->train_loaded = true;
+  return MF_OK;
+}
+
+static mf_status load_test(mf_ctx* c, int64_t N, const int32_t* u, const int32_t* v, const float* r,
+                           int on_device) {
+  const int32_t *du, *dv;
+  const float* dr;
+  int32_t *ou, *ov;
+  float* orr;
+  TRY(stage_input(c, N, u, v, r, on_device, &du, &dv, &dr, &ou, &ov, &orr));
+  TRY(validate(c, N, du, dv, dr));
+  TRY(c->alloc(&c->test, (size_t)std::max<int64_t>(N, 1)));
+  if (N > 0) {
+    k_build_test<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(du, dv, dr, N, c->rho_r, c->rho_c,
+                                                             (double)c->p.rating_scale, c->test);
+    KERNEL_TRY(c);
+  }
+  c->release(ou); c->release(ov); c->release(orr);
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  c->Ntest = N;
+  c->test_loaded = true;
+  return MF_OK;
+}
+
+mf_status mf_load_coo(mf_ctx* c, int32_t set, int64_t nnz, const int32_t* u, const int32_t* v,
+                      const float* r, int32_t on_device) {
+  if (!c) return MF_E_INVAL;
+  TRY(c->enter());
+  if (nnz < 0 || (nnz > 0 && (!u || !v || !r))) return c->fail(MF_E_INVAL, "bad COO arguments");
+  if (set == MF_TRAIN) {
+    if (c->train_loaded) return c->fail(MF_E_STATE, "train set already loaded");
+    return load_train(c, nnz, u, v, r, on_device);
+  }
+  if (set == MF_TEST) {
+    if (!c->train_loaded) return c->fail(MF_E_STATE, "load the train set first");
+    if (c->test_loaded) return c->fail(MF_E_STATE, "test set already loaded");
+    return load_test(c, nnz, u, v, r, on_device);
+  }
+  return c->fail(MF_E_INVAL, "set must be MF_TRAIN or MF_TEST");
+}
+
+// ---------------------------------------------------------------------------------------------
+// per-epoch schedule (A: "Orders")
+// ---------------------------------------------------------------------------------------------
+static mf_status build_schedule(mf_ctx* c, int32_t t) {
+  const int64_t nb = (int64_t)c->a * c->a;
+  if (!c->wf) {
+    const int64_t total = c->ch_off.back();
+    if (total == 0) return MF_OK;
+    k_chunk_keys<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(c->d_choff, (int)nb, c->p.seed, t,
+                                                                 c->sk0, c->sv0);
+    KERNEL_TRY(c);
+    ++c->n_launch;
+    if (nb == 1) {
+      TRY(c->sort_pairs(c->sk0, c->sk1, c->sv0, c->chunk_order, total, 64));
+    } else {
+      TRY(c->sort_pairs(c->sk0, c->sk1, c->sv0, c->sv1, total, 64));
+      k_chunk_block<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(c->sv1, c->d_choff, (int)nb,
+                                                                    total, c->sb);
+      KERNEL_TRY(c);
+      ++c->n_launch;
+      // stable by block: keeps each block's key order
+      uint32_t* bk_out = reinterpret_cast<uint32_t*>(c->sk0);
+      TRY(c->sort_pairs(c->sb, bk_out, c->sv1, c->chunk_order, total, bits_for((uint64_t)(nb - 1))));
+    }
+    c->sched_built_for = t;
+    return MF_OK;
+  }
+  // wavefront: seq (per block b, worker i: perm of c columns) then ticket ranks
+  const int s = c->s, cc = c->c;
+  const int64_t total = nb * s * (int64_t)cc;
+  if (c->p.cyclic) {
+    const int64_t tt = nb * cc;
+    for (int which = 0; which < 2; ++which) {
+      k_perm_keys<<<grid_for(tt, c->num_sms), 256, 0, c->st>>>(
+          nb, cc, c->p.seed, which == 0 ? kTagCycTau : kTagCycSigma, t, c->sk0, c->sv0);
+      KERNEL_TRY(c);
+      TRY(c->sort_pairs(c->sk0, c->sk1, c->sv0, c->sv1, tt, 64));
+      if (nb > 1) {
+        k_seg_of<<<grid_for(tt, c->num_sms), 256, 0, c->st>>>(c->sv1, tt, cc, c->sb);
+        KERNEL_TRY(c);
+        TRY(c->sort_pairs(c->sb, reinterpret_cast<uint32_t*>(c->sk0), c->sv1, c->sv0, tt,
+                          bits_for((uint64_t)(nb - 1))));
+        std::swap(c->sv0, c->sv1);
+      }
+      k_mod_c<<<grid_for(tt, c->num_sms), 256, 0, c->st>>>(c->sv1, tt, cc,
+                                                           which == 0 ? c->tau : c->sigma);
+      KERNEL_TRY(c);
+    }
+    k_cyclic_seq<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(c->tau, c->sigma, nb, s, cc, c->seq);
+    KERNEL_TRY(c);
+  } else {
+    k_wf_keys<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(nb * s, s, cc, c->p.seed, t, c->sk0,
+                                                              c->sv0);
+    KERNEL_TRY(c);
+    TRY(c->sort_pairs(c->sk0, c->sk1, c->sv0, c->sv1, total, 64));
+    if (nb * s > 1) {
+      k_seg_of<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(c->sv1, total, cc, c->sb);
+      KERNEL_TRY(c);
+      TRY(c->sort_pairs(c->sb, reinterpret_cast<uint32_t*>(c->sk0), c->sv1, c->sv0, total,
+                        bits_for((uint64_t)(nb * s - 1))));
+      std::swap(c->sv0, c->sv1);
+    }
+    k_mod_c<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(c->sv1, total, cc, c->seq);
+    KERNEL_TRY(c);
+  }
+  k_ticket_keys<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(c->seq, nb, s, cc, c->sk0, c->sv0);
+  KERNEL_TRY(c);
+  const uint64_t maxkey = (uint64_t)(((nb - 1) * cc + (cc - 1)) * (int64_t)cc + (cc - 1)) * s + (s - 1);
+  TRY(c->sort_pairs(c->sk0, c->sk1, c->sv0, c->sv1, total, bits_for(maxkey)));
+  k_ticket_rank<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(c->sv1, total, s, c->rank_arr);
+  KERNEL_TRY(c);
+  c->n_launch += 6;
+  c->sched_built_for = t;
+  return MF_OK;
+}
+
+static cudaEvent_t ev_at(mf_ctx* c, int i) {
+  while ((int)c->ev.size() <= i) {
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    c->ev.push_back(e);
+  }
+  return c->ev[(size_t)i];
+}
+
+// One strata block set (the blocks rank g trains in sub-epoch j) of epoch t.
+static mf_status run_stratum(mf_ctx* c, int32_t t, int j, const std::vector<int64_t>& pi, float g) {
+  std::vector<int64_t> blocks;
+  for (int r = c->lo_row_seg(); r < c->hi_row_seg(); ++r)
+    blocks.push_back((int64_t)r * c->a + (r + pi[(size_t)j]) % c->a);
+  if (!c->wf) {
+    ChunkSegs segs{};
+    segs.n = 0;
+    segs.prefix[0] = 0;
+    for (int64_t b : blocks) {
+      const int64_t nch = c->ch_off[(size_t)b + 1] - c->ch_off[(size_t)b];
+      if (nch == 0) continue;
+      segs.begin[segs.n] = c->ch_off[(size_t)b];
+      segs.prefix[segs.n + 1] = segs.prefix[segs.n] + nch;
+      c->updates += c->blk_len[(size_t)b];
+      ++segs.n;
+    }
+    if (segs.n == 0) return MF_OK;
+    CUDA_TRY(c, cudaMemsetAsync(c->counter, 0, sizeof(unsigned long long), c->st));
+    HogwildLaunch L{};
+    L.storage = c->p.storage; L.k = c->k; L.lane_bytes = c->p.lane_bytes ? c->p.lane_bytes : 16;
+    L.slots = c->slots; L.chunks = c->chunk_order; L.segs = segs; L.counter = c->counter;
+    L.workers = c->p.workers; L.num_sms = c->num_sms; L.f = c->f;
+    L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
+    L.out_workers = &c->last_workers; L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
+    CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
+    CUDA_TRY(c, launch_hogwild(L));
+    CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd + 1), c->st));
+    c->last_block = 256;
+    ++c->n_sgd;
+    ++c->n_launch;
+    return MF_OK;
+  }
+  for (int64_t b : blocks) {
+    if (c->blk_len[(size_t)b] == 0) continue;
+    CUDA_TRY(c, cudaMemsetAsync(c->tickets, 0, (size_t)c->c * 4, c->st));
+    const int64_t base = b * (int64_t)c->s * c->c;
+    WavefrontLaunch L{};
+    L.storage = c->p.storage; L.k = c->k; L.slots = c->slots; L.sub_off = c->sub_off + base;
+    L.seq = c->seq + base; L.rank = c->rank_arr + base; L.tickets = c->tickets;
+    L.s = c->s; L.c = c->c; L.num_sms = c->num_sms; L.P = c->P; L.Q = c->Q; L.g = g;
+    L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
+    L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
+    CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
+    cudaError_t e = launch_wavefront(L);
+    if (e == cudaErrorCooperativeLaunchTooLarge) {
+      cudaGetLastError();
+      return c->fail(MF_E_UNSUPPORTED, "wavefront: %d workers cannot all be co-resident", c->s);
+    }
+    CUDA_TRY(c, e);
+    CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd + 1), c->st));
+    c->last_workers = c->s;
+    c->last_block = 128;
+    c->updates += c->blk_len[(size_t)b];
+    ++c->n_sgd;
+    ++c->n_launch;
+  }
+  return MF_OK;
+}
+
+// Q segment J occupies relabelled rows [ceil(J n / a), ceil((J+1) n / a)) (A: segments).
+static void q_segment(const mf_ctx* c, int J, char** ptr, size_t* bytes) {
+  const size_t row_bytes = (size_t)c->k * c->ssize();
+  const int64_t lo = cdiv64((int64_t)J * c->n, c->a), hi = cdiv64((int64_t)(J + 1) * c->n, c->a);
+  *ptr = (char*)c->Q + (size_t)lo * row_bytes;
+  *bytes = (size_t)(hi - lo) * row_bytes;
+}
+
+// Move every Q segment whose holder changes from `from` to `to` (north_star (5): NCCL
+// send/recv of Q column-segments between sub-epochs).  from[J] < 0: every rank already holds
+// a valid copy, nothing moves.
+static mf_status rotate_q(mf_ctx* c, const int32_t* from, const int32_t* to) {
+  if (c->G == 1) return MF_OK;
+  std::vector<mf::Xfer> xs;
+  for (int J = 0; J < c->a; ++J) {
+    if (from[J] < 0 || from[J] == to[J]) continue;
+    mf::Xfer x;
+    q_segment(c, J, (char**)&x.ptr, &x.bytes);
+    x.src = from[J];
+    x.dst = to[J];
+    xs.push_back(x);
+  }
+  std::string why;
+  if (!c->comm->exchange(xs, c->rank, &why)) return c->fail(MF_E_NCCL, "Q rotation: %s", why.c_str());
+  return MF_OK;
+}
+
+// Make every rank's Q complete (evaluation / get_factors): broadcast each segment from its
+// current holder; afterwards every rank holds an identical valid copy (holders = -1).
+static mf_status gather_q(mf_ctx* c) {
+  if (c->G == 1) return MF_OK;
+  const int32_t* h = c->comm->holders(c->a);
+  std::vector<int32_t> hold(h, h + c->a);
+  for (int J = 0; J < c->a; ++J) {
+    if (hold[(size_t)J] < 0) continue;
+    char* ptr;
+    size_t bytes;
+    q_segment(c, J, &ptr, &bytes);
+    std::string why;
+    if (!c->comm->broadcast(ptr, bytes, hold[(size_t)J], &why))
+      return c->fail(MF_E_NCCL, "Q gather: %s", why.c_str());
+  }
+  c->comm->reset_holders(c->a);
+  return MF_OK;
+}
+
+mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
+  if (!c) return MF_E_INVAL;
+  TRY(c->enter());
+  if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
+  const int32_t t = c->t;
+  const float g = gamma_of(c->p.alpha, c->p.beta, t);   // Eq. 9
+  c->n_sgd = 0;
+  c->n_launch = 0;
+  c->updates = 0;
+  c->comm_ms_acc.clear();
+  CUDA_TRY(c, cudaEventRecord(c->ev_e0, c->st));
+  CUDA_TRY(c, cudaEventRecord(c->ev_s0, c->st));
+  TRY(build_schedule(c, t));
+  CUDA_TRY(c, cudaEventRecord(c->ev_s1, c->st));
+  const std::vector<int64_t> pi = host_perm(make_stream(c->p.seed, kTagStrata, (uint64_t)t, 0), c->a);
+  std::vector<int32_t> hold((size_t)c->a), next((size_t)c->a);
+  CUDA_TRY(c, cudaEventRecord(c->ev_c0, c->st));
+  CUDA_TRY(c, cudaEventRecord(c->ev_c1, c->st));
+  for (int j = 0; j < c->a; ++j) {
+    if (c->G > 1) {
+      // before sub-epoch j: move every segment whose holder changes (holders of the previous
+      // sub-epoch -- or of the previous epoch's last one -- are tracked in comm)
+      mf_strata_holders(c->p.seed, c->a, c->G, t, j, next.data());
+      TRY(rotate_q(c, c->comm->holders(c->a), next.data()));
+      c->comm->set_holders(next.data(), c->a);
+    }
+    TRY(run_stratum(c, t, j, pi, g));
+  }
+  CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
+  c->t = t + 1;
+  c->have_stats = true;
+  if (epoch_done) *epoch_done = c->t;
+  return MF_OK;
+}
+
+mf_status mf_get_stats(mf_ctx* c, mf_stats* out) {
+  if (!c || !out) return MF_E_INVAL;
+  TRY(c->enter());
+  std::memset(out, 0, sizeof *out);
+  if (!c->have_stats) return MF_OK;
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  float ms = 0.f;
+  CUDA_TRY(c, cudaEventElapsedTime(&ms, c->ev_e0, c->ev_e1));
+  out->epoch_ms = ms;
+  CUDA_TRY(c, cudaEventElapsedTime(&ms, c->ev_s0, c->ev_s1));
+  out->sched_ms = ms;
+  double sgd = 0.0;
+  for (int i = 0; i < c->n_sgd; ++i) {
+    CUDA_TRY(c, cudaEventElapsedTime(&ms, c->ev[(size_t)(2 * i)], c->ev[(size_t)(2 * i + 1)]));
+    sgd += ms;
+  }
+  out->sgd_ms = sgd;
+  out->comm_ms = std::max(0.0, out->epoch_ms - out->sched_ms - sgd);
+  out->sgd_launches = c->n_sgd;
+  out->launches = c->n_launch;
+  out->updates = c->updates;
+  out->bytes_per_update = 12 + 4 * (int64_t)c->k * c->ssize();
+  out->workers = c->last_workers;
+  out->lanes = c->last_lanes;
+  out->grid = c->last_grid;
+  out->block = c->last_block;
+  return MF_OK;
+}
+
+// ---------------------------------------------------------------------------------------------
+// rmse / factors
+// ---------------------------------------------------------------------------------------------
+mf_status mf_rmse(mf_ctx* c, int32_t set, double* out) {
+  if (!c || !out) return MF_E_INVAL;
+  TRY(c->enter());
+  if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
+  const Rating* data;
+  int64_t N;
+  if (set == MF_TEST) {
+    if (!c->test_loaded) return c->fail(MF_E_STATE, "no test set loaded");
+    data = c->test;
+    N = c->Ntest;
+  } else if (set == MF_TRAIN) {
+    data = c->slots;  // sentinel pad slots (u < 0) are skipped by the kernel
+    N = c->nslots;
+  } else {
+    return c->fail(MF_E_INVAL, "bad set");
+  }
+  if (set == MF_TRAIN && c->G > 1)
+    return c->fail(MF_E_UNSUPPORTED, "train-set RMSE is single-GPU only");
+  // world > 1: every rank evaluates the test samples of the row segments it owns (filtered at
+  // load) against a complete Q, then the SSE and count are summed over ranks.
+  if (c->G > 1) TRY(gather_q(c));
+  RmseLaunch L{};
+  L.storage = c->p.storage; L.k = c->k; L.test = data; L.N = N; L.P = c->P; L.Q = c->Q;
+  L.partial = c->rm_partial; L.out = c->rm_out; L.num_sms = c->num_sms; L.stream = c->st;
+  CUDA_TRY(c, launch_rmse(L));
+  double cnt = (double)(set == MF_TRAIN ? c->N : N);
+  if (c->G > 1) {
+    CUDA_TRY(c, cudaMemcpyAsync(c->rm_out + 1, &cnt, 8, cudaMemcpyHostToDevice, c->st));
+    std::string why;
+    if (!c->comm->allreduce_sum(c->rm_out, 2, &why)) return c->fail(MF_E_NCCL, "rmse: %s", why.c_str());
+  }
+  double h2[2] = {0.0, 0.0};
+  CUDA_TRY(c, cudaMemcpyAsync(h2, c->rm_out, 16, cudaMemcpyDeviceToHost, c->st));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  const double sse = h2[0];
+  if (c->G > 1) cnt = h2[1];
+  const double rmse = (double)c->p.rating_scale * std::sqrt(sse / std::max(cnt, 1.0));
+  *out = N > 0 ? rmse : 0.0;
+  if (std::isnan(*out)) return c->fail(MF_E_RANGE, "RMSE is NaN (divergence)");
+  return MF_OK;
+}
+
+template <typename T>
+static void unrelabel_t(mf_ctx* c, const void* X, const int32_t* rho, int64_t rows, float* out) {
+  k_unrelabel<T><<<grid_for(rows * c->k, c->num_sms), 256, 0, c->st>>>((const T*)X, rho, rows, c->k, out);
+}
+template <typename T>
+static void relabel_store_t(mf_ctx* c, void* X, const int32_t* rho, int64_t rows, const float* in) {
+  k_relabel_store<T><<<grid_for(rows * c->k, c->num_sms), 256, 0, c->st>>>((T*)X, rho, rows, c->k, in);
+}
+
+static mf_status get_one(mf_ctx* c, const void* X, const int32_t* rho, int64_t rows, float* dst,
+                         int on_device) {
+  float* d = dst;
+  if (!on_device) TRY(c->alloc(&d, (size_t)(rows * c->k)));
+  switch (c->p.storage) {
+    case MF_FP32: unrelabel_t<float>(c, X, rho, rows, d); break;
+    case MF_FP16: unrelabel_t<__half>(c, X, rho, rows, d); break;
+    default: unrelabel_t<__nv_bfloat16>(c, X, rho, rows, d); break;
+  }
+  KERNEL_TRY(c);
+  if (!on_device) {
+    CUDA_TRY(c, cudaMemcpyAsync(dst, d, (size_t)(rows * c->k) * 4, cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    c->release(d);
+  }
+  return MF_OK;
+}
+
+mf_status mf_get_factors(mf_ctx* c, float* P, float* Q, int32_t on_device) {
+  if (!c) return MF_E_INVAL;
+  TRY(c->enter());
+  if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
+  if (c->G > 1) {
+    TRY(gather_q(c));
+    std::string why;
+    const size_t row_bytes = (size_t)c->k * c->ssize();
+    if (!c->comm->gather_rows(c->P, c->m, c->a, c->G, row_bytes, &why))
+      return c->fail(MF_E_NCCL, "P gather: %s", why.c_str());
+  }
+  if (P) TRY(get_one(c, c->P, c->rho_r, c->m, P, on_device));
+  if (Q) TRY(get_one(c, c->Q, c->rho_c, c->n, Q, on_device));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  return MF_OK;
+}
+
+static mf_status set_one(mf_ctx* c, void* X, const int32_t* rho, int64_t rows, const float* src,
+                         int on_device) {
+  const float* d = src;
+  float* own = nullptr;
+  if (!on_device) {
+    TRY(c->alloc(&own, (size_t)(rows * c->k)));
+    CUDA_TRY(c, cudaMemcpyAsync(own, src, (size_t)(rows * c->k) * 4, cudaMemcpyHostToDevice, c->st));
+    d = own;
+  }
+  switch (c->p.storage) {
+    case MF_FP32: relabel_store_t<float>(c, X, rho, rows, d); break;
+    case MF_FP16: relabel_store_t<__half>(c, X, rho, rows, d); break;
+    default: relabel_store_t<__nv_bfloat16>(c, X, rho, rows, d); break;
+  }
+  KERNEL_TRY(c);
+  if (own) {
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    c->release(own);
+  }
+  return MF_OK;
+}
+
+mf_status mf_set_factors(mf_ctx* c, const float* P, const float* Q, int32_t on_device) {
+  if (!c) return MF_E_INVAL;
+  TRY(c->enter());
+  if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
+  if (P) TRY(set_one(c, c->P, c->rho_r, c->m, P, on_device));
+  if (Q) TRY(set_one(c, c->Q, c->rho_c, c->n, Q, on_device));
+  if (c->G > 1 && Q) c->comm->reset_holders(c->a);  // every rank holds a valid copy again
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  return MF_OK;
+}
+
+mf_status mf_set_epoch(mf_ctx* c, int32_t t) {
+  if (!c || t < 0) return MF_E_INVAL;
+  c->t = t;
+  return MF_OK;
+}
+mf_status mf_get_epoch(const mf_ctx* c, int32_t* t) {
+  if (!c || !t) return MF_E_INVAL;
+  *t = c->t;
+  return MF_OK;
+}
+
+// ---------------------------------------------------------------------------------------------
+// exports
+// ---------------------------------------------------------------------------------------------
+template <typename X>
+static mf_status d2h(mf_ctx* c, std::vector<X>& h, const X* d, int64_t n) {
+  h.resize((size_t)std::max<int64_t>(n, 1));
+  if (n > 0) CUDA_TRY(c, cudaMemcpyAsync(h.data(), d, (size_t)n * sizeof(X), cudaMemcpyDeviceToHost, c->st));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  return MF_OK;
+}
+
+mf_status mf_export_schedule(mf_ctx* c, int32_t what, int32_t epoch, int64_t* buf, int64_t* len) {
+  if (!c || !len) return MF_E_INVAL;
+  TRY(c->enter());
+  if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
+  const int64_t nb = (int64_t)c->a * c->a;
+  int64_t need = 0;
+  switch (what) {
+    case MF_EX_PERM: case MF_EX_BLOCKID: need = c->N; break;
+    case MF_EX_RHO_R: need = c->m; break;
+    case MF_EX_RHO_C: need = c->n; break;
+    case MF_EX_CHUNKORDER:
+      if (c->wf) return c->fail(MF_E_INVAL, "no chunk order in wavefront mode");
+      need = c->ch_off.back();
+      break;
+    case MF_EX_WFSEQ: case MF_EX_TICKETS:
+      if (!c->wf) return c->fail(MF_E_INVAL, "no wavefront schedule in Hogwild mode");
+      need = nb * c->s * (int64_t)c->c;
+      break;
+    case MF_EX_STRATA: need = c->a; break;
+    default: return c->fail(MF_E_INVAL, "unknown export %d", what);
+  }
+  if (!buf) { *len = need; return MF_OK; }
+  if (*len < need) return c->fail(MF_E_INVAL, "buffer too small (%lld < %lld)", (long long)*len, (long long)need);
+  *len = need;
+  switch (what) {
+    case MF_EX_PERM: {
+      std::vector<uint32_t> h;
+      TRY(d2h(c, h, c->perm, c->N));
+      for (int64_t j = 0; j < c->N; ++j) buf[j] = h[(size_t)j];
+      return MF_OK;
+    }
+    case MF_EX_RHO_R: case MF_EX_RHO_C: {
+      std::vector<int32_t> h;
+      const int64_t n = what == MF_EX_RHO_R ? c->m : c->n;
+      TRY(d2h(c, h, what == MF_EX_RHO_R ? c->rho_r : c->rho_c, n));
+      for (int64_t j = 0; j < n; ++j) buf[j] = h[(size_t)j];
+      return MF_OK;
+    }
+    case MF_EX_BLOCKID: {
+      std::vector<uint32_t> pos;
+      TRY(d2h(c, pos, c->slot_pos, c->nslots));
+      if (!c->wf) {
+        for (int64_t b = 0; b < nb; ++b)
+          for (int64_t x = c->blk_off[(size_t)b]; x < c->blk_off[(size_t)b] + c->blk_len[(size_t)b]; ++x)
+            buf[pos[(size_t)x]] = b;
+      } else {
+        std::vector<int64_t> off;
+        TRY(d2h(c, off, c->sub_off, nb * c->s * (int64_t)c->c + 1));
+        for (int64_t q = 0; q < nb * c->s * (int64_t)c->c; ++q)
+          for (int64_t x = off[(size_t)q]; x < off[(size_t)q + 1]; ++x) buf[pos[(size_t)x]] = q;
+      }
+      return MF_OK;
+    }
+    case MF_EX_CHUNKORDER: {
+      TRY(build_schedule(c, epoch));
+      std::vector<uint32_t> h;
+      TRY(d2h(c, h, c->chunk_order, need));
+      for (int64_t b = 0; b < nb; ++b)
+        for (int64_t x = c->ch_off[(size_t)b]; x < c->ch_off[(size_t)b + 1]; ++x)
+          buf[x] = (int64_t)h[(size_t)x] - c->ch_off[(size_t)b];
+      return MF_OK;
+    }
+    case MF_EX_WFSEQ: case MF_EX_TICKETS: {
+      TRY(build_schedule(c, epoch));
+      std::vector<int32_t> h;
+      TRY(d2h(c, h, what == MF_EX_WFSEQ ? c->seq : c->rank_arr, need));
+      for (int64_t x = 0; x < need; ++x) buf[x] = h[(size_t)x];
+      return MF_OK;
+    }
+    case MF_EX_STRATA: {
+      std::vector<int64_t> pi = host_perm(make_stream(c->p.seed, kTagStrata, (uint64_t)epoch, 0), c->a);
+      for (int64_t x = 0; x < c->a; ++x) buf[x] = pi[(size_t)x];
+      return MF_OK;
+    }
+  }
+  return MF_E_INVAL;
+}
+

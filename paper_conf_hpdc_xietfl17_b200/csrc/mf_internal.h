@@ -1,0 +1,63 @@
+// mf_internal.h -- internal launch descriptors shared by mf_api.cu, mf_prep.cu, mf_kernels.cu.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "mf_common.cuh"
+
+namespace mfb {
+
+constexpr int kMaxSegs = 8;  // blocks per Hogwild launch (a/G <= 8 strata blocks)
+
+// Chunk list of one Hogwild launch: segment s is chunks[begin[s] .. begin[s] + prefix[s+1]-prefix[s]).
+struct ChunkSegs {
+  int64_t begin[kMaxSegs];
+  int64_t prefix[kMaxSegs + 1];
+  int n;
+};
+
+struct HogwildLaunch {
+  int storage, k, lane_bytes;
+  const Rating* slots;
+  const uint32_t* chunks;
+  ChunkSegs segs;
+  unsigned long long* counter;
+  int workers, num_sms, f;
+  void *P, *Q;
+  float g, lp, lq;
+  cudaStream_t stream;
+  int *out_workers, *out_lanes, *out_grid;
+};
+
+struct WavefrontLaunch {
+  int storage, k;
+  const Rating* slots;
+  const int64_t* sub_off;  // s*c + 1 slot offsets of this strata block's sub-blocks
+  const int32_t* seq;      // s*c
+  const int32_t* rank;     // s*c
+  int* tickets;            // c
+  int s, c, num_sms;
+  void *P, *Q;
+  float g, lp, lq;
+  cudaStream_t stream;
+  int *out_lanes, *out_grid;
+};
+
+struct RmseLaunch {
+  int storage, k;
+  const Rating* test;
+  int64_t N;
+  const void *P, *Q;
+  double* partial;  // num_sms*4
+  double* out;      // 1
+  int num_sms;
+  cudaStream_t stream;
+};
+
+cudaError_t launch_hogwild(const HogwildLaunch& a);
+cudaError_t launch_wavefront(const WavefrontLaunch& a);
+cudaError_t launch_rmse(const RmseLaunch& a);
+
+}  // namespace mfb

@@ -1,0 +1,279 @@
+// mf_kernels.cu -- SGD kernels (batch-Hogwild!, wavefront) and the RMSE kernel, with the
+// runtime dispatch over (k, storage, lanes) template instantiations.
+#include <cuda_runtime.h>
+
+#include "mf_internal.h"
+#include "mf_sgd.cuh"
+
+namespace mfb {
+
+// ---------------------------------------------------------------------------------------------
+// batch-Hogwild! (section 5.1).  A worker is a group of L lanes; a warp holds
+// 32/L workers which claim consecutive entries of the epoch's chunk list with ONE atomicAdd per
+// warp (the only scheduling synchronisation, "lock-free"), then each worker updates the
+// f consecutive slots of its chunk serially.  Persistent grid: workers loop until the list is
+// exhausted.  The chunk list of a launch is the concatenation of up to kMaxSegs block segments.
+// ---------------------------------------------------------------------------------------------
+template <typename T, int K, int L>
+__global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slots,
+                                                 const uint32_t* __restrict__ chunks, ChunkSegs segs,
+                                                 unsigned long long* __restrict__ counter,
+                                                 int workers, T* __restrict__ P, T* __restrict__ Q,
+                                                 int f, float g, float lp, float lq) {
+  constexpr int GPW = 32 / L;
+  const int lane = threadIdx.x & 31;
+  const int grp = lane / L, gl = lane % L, gbase = grp * L;
+  const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
+  const int warp = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) >> 5);
+  const int first = warp * GPW;
+  if (first >= workers) return;                      // warp-uniform
+  const int nact = min(GPW, workers - first);
+  const int64_t total = segs.prefix[segs.n];
+  for (;;) {
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(counter, (unsigned long long)nact);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if ((int64_t)base >= total) break;
+    const int64_t ci = (int64_t)base + grp;
+    int64_t lo = 0, hi = 0;
+    if (grp < nact && ci < total) {
+      int sgi = 0;
+      while (ci >= segs.prefix[sgi + 1]) ++sgi;
+      const uint32_t chunk = __ldg(chunks + segs.begin[sgi] + (ci - segs.prefix[sgi]));
+      lo = (int64_t)chunk * f;
+      hi = lo + f;
+    }
+    run_serial<T, K, L>(slots, lo, hi, P, Q, g, lp, lq, gl, gbase, gmask);
+  }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Wavefront (section 5.2, Fig. 6).  Worker i (a group of L lanes) owns row
+// sub-block i and walks its column sequence seq_i[0..c).  Before wave w it waits on the 1-D
+// column array ("column lock array") until the column's ticket equals the precomputed
+// rank of visit (w,i) (R10: deterministic (w,i)-lexicographic tie-break), runs the sub-block
+// serially, and releases the column with ticket+1.  Every wait is on a lexicographically
+// smaller visit, so with all workers co-resident (cooperative launch) there is no deadlock.
+// ---------------------------------------------------------------------------------------------
+__device__ __forceinline__ int ld_acquire(const int* p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(int* p, int v) {
+  asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+template <typename T, int K, int L>
+__global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ slots,
+                                                   const int64_t* __restrict__ sub_off,
+                                                   const int32_t* __restrict__ seq,
+                                                   const int32_t* __restrict__ rank,
+                                                   int* __restrict__ tickets, int s, int c,
+                                                   T* __restrict__ P, T* __restrict__ Q, float g,
+                                                   float lp, float lq) {
+  const int lane = threadIdx.x & 31;
+  const int grp = lane / L, gl = lane % L, gbase = grp * L;
+  const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
+  const int worker = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) / L);
+  if (worker >= s) return;
+  const int32_t* my_seq = seq + (int64_t)worker * c;
+  const int32_t* my_rank = rank + (int64_t)worker * c;
+  for (int w = 0; w < c; ++w) {
+    const int col = __ldg(my_seq + w);
+    const int tgt = __ldg(my_rank + w);
+    while (ld_acquire(tickets + col) != tgt) __nanosleep(64);
+    const int64_t sb = (int64_t)worker * c + col;
+    run_serial<T, K, L>(slots, __ldg(sub_off + sb), __ldg(sub_off + sb + 1), P, Q, g, lp, lq, gl,
+                        gbase, gmask);
+    __threadfence();
+    __syncwarp(gmask);
+    if (gl == 0) st_release(tickets + col, tgt + 1);
+  }
+}
+
+// ---------------------------------------------------------------------------------------------
+// RMSE (R13): per-group fp32 dot, per-lane-0 fp64 accumulation, fixed-order block
+// reduction to one partial per CTA; k_rmse_final sums the partials in a fixed order.
+// ---------------------------------------------------------------------------------------------
+template <typename T, int K, int L>
+__global__ void __launch_bounds__(256) k_rmse_partial(const Rating* __restrict__ test, int64_t N,
+                                                      const T* __restrict__ P,
+                                                      const T* __restrict__ Q,
+                                                      double* __restrict__ partial) {
+  using G = Geo<T, K, L>;
+  constexpr int PW = Pack<T>::kPerWord;
+  const int lane = threadIdx.x & 31;
+  const int grp = lane / L, gl = lane % L, gbase = grp * L;
+  const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
+  const int gpb = blockDim.x / L;
+  const int64_t stride = (int64_t)gridDim.x * gpb;
+  double acc = 0.0;
+  for (int64_t x = (int64_t)blockIdx.x * gpb + threadIdx.x / L; x < N; x += stride) {
+    const int* tp = reinterpret_cast<const int*>(test + x);
+    const int u = __ldcs(tp), v = __ldcs(tp + 1);
+    const float r = __int_as_float(__ldcs(tp + 2));
+    if (u < 0) continue;  // sentinel pad slot (group-uniform)
+    Words<G::NW> pw, qw;
+    load_row(row_ptr<T, K>(P, u, gl, G::VEC), pw);
+    load_row(row_ptr<T, K>(Q, v, gl, G::VEC), qw);
+    float p[G::VEC], q[G::VEC];
+#pragma unroll
+    for (int i = 0; i < G::NW; ++i) {
+      Pack<T>::unpack(pw.w[i], p + i * PW);
+      Pack<T>::unpack(qw.w[i], q + i * PW);
+    }
+    float d = 0.f;
+#pragma unroll
+    for (int e = 0; e < G::VEC; ++e) d = fmaf(p[e], q[e], d);
+#pragma unroll
+    for (int o = L / 2; o > 0; o >>= 1) d += __shfl_xor_sync(gmask, d, o);
+    const float e = r - d;
+    if (gl == 0) acc += (double)e * (double)e;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  __shared__ double wsum[32];
+  if (lane == 0) wsum[threadIdx.x >> 5] = acc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double s = 0.0;
+    for (int i = 0; i < (int)(blockDim.x >> 5); ++i) s += wsum[i];
+    partial[blockIdx.x] = s;
+  }
+}
+
+__global__ void k_rmse_final(const double* __restrict__ partial, int n, double* __restrict__ out) {
+  __shared__ double sm[256];
+  double s = 0.0;
+  for (int i = threadIdx.x; i < n; i += blockDim.x) s += partial[i];
+  sm[threadIdx.x] = s;
+  __syncthreads();
+  for (int w = blockDim.x / 2; w > 0; w >>= 1) {
+    if ((int)threadIdx.x < w) sm[threadIdx.x] += sm[threadIdx.x + w];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) out[0] = sm[0];
+}
+
+// ---------------------------------------------------------------------------------------------
+// Dispatch
+// ---------------------------------------------------------------------------------------------
+template <typename T, int K, int L>
+static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
+  auto kern = k_hogwild<T, K, L>;
+  const int threads = 256;
+  int per_sm = 0;
+  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, 0);
+  if (e != cudaSuccess) return e;
+  const int gpw = 32 / L;
+  const int resident_workers = per_sm * a.num_sms * (threads / 32) * gpw;
+  int workers = a.workers > 0 ? a.workers : resident_workers;
+  int blocks = (int)cdiv64((int64_t)workers, (int64_t)(threads / 32) * gpw);
+  if (a.out_workers) *a.out_workers = workers;
+  if (a.out_lanes) *a.out_lanes = L;
+  if (a.out_grid) *a.out_grid = blocks;
+  kern<<<blocks, threads, 0, a.stream>>>(a.slots, a.chunks, a.segs, a.counter, workers,
+                                         reinterpret_cast<T*>(a.P), reinterpret_cast<T*>(a.Q), a.f,
+                                         a.g, a.lp, a.lq);
+  return cudaGetLastError();
+}
+
+template <typename T, int K, int L>
+static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
+  auto kern = k_wavefront<T, K, L>;
+  const int threads = 128;
+  const int64_t total_threads = (int64_t)a.s * L;
+  const int blocks = (int)cdiv64(total_threads, threads);
+  int per_sm = 0;
+  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, 0);
+  if (e != cudaSuccess) return e;
+  if ((int64_t)per_sm * a.num_sms < blocks) return cudaErrorCooperativeLaunchTooLarge;
+  if (a.out_lanes) *a.out_lanes = L;
+  if (a.out_grid) *a.out_grid = blocks;
+  const Rating* slots = a.slots;
+  const int64_t* sub_off = a.sub_off;
+  const int32_t* seq = a.seq;
+  const int32_t* rank = a.rank;
+  int* tickets = a.tickets;
+  int s = a.s, c = a.c;
+  T* P = reinterpret_cast<T*>(a.P);
+  T* Q = reinterpret_cast<T*>(a.Q);
+  float g = a.g, lp = a.lp, lq = a.lq;
+  void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq};
+  return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, 0,
+                                     a.stream);
+}
+
+template <typename T, int K, int L>
+static cudaError_t launch_rmse_t(const RmseLaunch& a) {
+  const int threads = 256;
+  const int blocks = a.num_sms * 4;
+  if (a.N > 0)
+    k_rmse_partial<T, K, L><<<blocks, threads, 0, a.stream>>>(
+        a.test, a.N, reinterpret_cast<const T*>(a.P), reinterpret_cast<const T*>(a.Q), a.partial);
+  else
+    cudaMemsetAsync(a.partial, 0, sizeof(double) * blocks, a.stream);
+  k_rmse_final<<<1, 256, 0, a.stream>>>(a.partial, blocks, a.out);
+  return cudaGetLastError();
+}
+
+// lanes per sample for a given bytes-per-lane target: L = clamp(k*S/lane_bytes, 1, 32)
+static constexpr int lanes_for(int K, int S, int LB) {
+  return (K * S / LB) >= 32 ? 32 : ((K * S / LB) < 1 ? 1 : (K * S / LB));
+}
+
+template <typename T, int K>
+static cudaError_t hogwild_k(const HogwildLaunch& a) {
+  constexpr int S = (int)sizeof(T);
+  if (a.lane_bytes == 32) return launch_hogwild_t<T, K, lanes_for(K, S, 32)>(a);
+  return launch_hogwild_t<T, K, lanes_for(K, S, 16)>(a);
+}
+template <typename T, int K>
+static cudaError_t rmse_k(const RmseLaunch& a) {
+  constexpr int S = (int)sizeof(T);
+  return launch_rmse_t<T, K, lanes_for(K, S, 16)>(a);
+}
+template <typename T, int K>
+static cudaError_t wavefront_k(const WavefrontLaunch& a) {
+  constexpr int S = (int)sizeof(T);
+  return launch_wavefront_t<T, K, lanes_for(K, S, 8)>(a);
+}
+
+#define MF_DISPATCH(FN, ARG)                                                         \
+  switch (ARG.storage) {                                                             \
+    case 0:                                                                          \
+      switch (ARG.k) {                                                               \
+        case 16: return FN<float, 16>(ARG);                                          \
+        case 32: return FN<float, 32>(ARG);                                          \
+        case 64: return FN<float, 64>(ARG);                                          \
+        case 128: return FN<float, 128>(ARG);                                        \
+        case 256: return FN<float, 256>(ARG);                                        \
+      }                                                                              \
+      break;                                                                         \
+    case 1:                                                                          \
+      switch (ARG.k) {                                                               \
+        case 16: return FN<__half, 16>(ARG);                                         \
+        case 32: return FN<__half, 32>(ARG);                                         \
+        case 64: return FN<__half, 64>(ARG);                                         \
+        case 128: return FN<__half, 128>(ARG);                                       \
+        case 256: return FN<__half, 256>(ARG);                                       \
+      }                                                                              \
+      break;                                                                         \
+    case 2:                                                                          \
+      switch (ARG.k) {                                                               \
+        case 16: return FN<__nv_bfloat16, 16>(ARG);                                  \
+        case 32: return FN<__nv_bfloat16, 32>(ARG);                                  \
+        case 64: return FN<__nv_bfloat16, 64>(ARG);                                  \
+        case 128: return FN<__nv_bfloat16, 128>(ARG);                                \
+        case 256: return FN<__nv_bfloat16, 256>(ARG);                                \
+      }                                                                              \
+      break;                                                                         \
+  }                                                                                  \
+  return cudaErrorInvalidValue;
+
+cudaError_t launch_hogwild(const HogwildLaunch& a) { MF_DISPATCH(hogwild_k, a) }
+cudaError_t launch_wavefront(const WavefrontLaunch& a) { MF_DISPATCH(wavefront_k, a) }
+cudaError_t launch_rmse(const RmseLaunch& a) { MF_DISPATCH(rmse_k, a) }
+
+}  // namespace mfb

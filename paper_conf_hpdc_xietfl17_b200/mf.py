@@ -1,0 +1,325 @@
+"""ctypes binding of libmf_b200.so (include/mf.h): argument marshalling only.
+
+Every step of the hot path runs in the library's CUDA kernels.  There is no CPU fallback:
+if the library is missing or the device is unavailable, the calls raise.  PyTorch is used for
+device memory (the optional caching-allocator hooks), streams (``torch.cuda.current_stream``)
+and, in the multi-GPU mode, the process group that broadcasts the ncclUniqueId.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libmf_b200.so")
+
+STORAGE = {"fp32": 0, "fp16": 1, "bf16": 2}
+SCHEDULE = {"hogwild": 0, "wavefront": 1}
+SETS = {"train": 0, "test": 1}
+EXPORTS = {"perm": 0, "rho_r": 1, "rho_c": 2, "blockid": 3, "chunkorder": 4, "wfseq": 5,
+           "tickets": 6, "strata": 7}
+STATUS = {0: "MF_OK", -1: "MF_E_INVAL", -2: "MF_E_NOMEM", -3: "MF_E_CUDA", -4: "MF_E_NCCL",
+          -5: "MF_E_STATE", -6: "MF_E_RANGE", -7: "MF_E_UNSUPPORTED"}
+
+
+class MFError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+
+
+class Allocator(ctypes.Structure):
+    _fields_ = [("alloc", _ALLOC_FN), ("free", _FREE_FN), ("user", ctypes.c_void_p)]
+
+
+class Params(ctypes.Structure):
+    _fields_ = [("struct_size", ctypes.c_uint32), ("m", ctypes.c_int64), ("n", ctypes.c_int64),
+                ("k", ctypes.c_int32), ("lambda_p", ctypes.c_float), ("lambda_q", ctypes.c_float),
+                ("alpha", ctypes.c_float), ("beta", ctypes.c_float),
+                ("init_scale", ctypes.c_float), ("rating_scale", ctypes.c_float),
+                ("seed", ctypes.c_uint64), ("schedule", ctypes.c_int32),
+                ("storage", ctypes.c_int32), ("workers", ctypes.c_int32),
+                ("batch_f", ctypes.c_int32), ("wf_cols", ctypes.c_int32),
+                ("grid_a", ctypes.c_int32), ("cyclic", ctypes.c_int32),
+                ("lane_bytes", ctypes.c_int32), ("device", ctypes.c_int32),
+                ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("transport", ctypes.c_int32), ("nccl_id", ctypes.c_void_p),
+                ("stream", ctypes.c_void_p), ("alloc", ctypes.POINTER(Allocator))]
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [("epoch_ms", ctypes.c_double), ("sgd_ms", ctypes.c_double),
+                ("sched_ms", ctypes.c_double), ("comm_ms", ctypes.c_double),
+                ("sgd_launches", ctypes.c_int64), ("launches", ctypes.c_int64),
+                ("updates", ctypes.c_int64), ("bytes_per_update", ctypes.c_int64),
+                ("workers", ctypes.c_int32), ("lanes", ctypes.c_int32),
+                ("grid", ctypes.c_int32), ("block", ctypes.c_int32)]
+
+
+_lib = None
+EXPORTED = ["mf_abi_version", "mf_params_default", "mf_create", "mf_load_coo", "mf_train_epoch",
+            "mf_rmse", "mf_get_factors", "mf_set_factors", "mf_set_epoch", "mf_get_epoch",
+            "mf_export_schedule", "mf_get_stats", "mf_strata_holders", "mf_destroy",
+            "mf_last_error", "mf_status_string"]
+
+
+def lib() -> ctypes.CDLL:
+    """Load libmf_b200.so (raises if it has not been built: no fallback path exists)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is not built; run `python -m paper_conf_hpdc_xietfl17_b200.build`"
+                          " (the CUDA path has no CPU fallback)")
+    L = ctypes.CDLL(LIB_PATH)
+    i32, i64, u64, vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64, ctypes.c_void_p
+    sig = {
+        "mf_abi_version": (i32, []),
+        "mf_params_default": (i32, [ctypes.POINTER(Params)]),
+        "mf_create": (i32, [ctypes.POINTER(Params), ctypes.POINTER(vp)]),
+        "mf_load_coo": (i32, [vp, i32, i64, vp, vp, vp, i32]),
+        "mf_train_epoch": (i32, [vp, ctypes.POINTER(i32)]),
+        "mf_rmse": (i32, [vp, i32, ctypes.POINTER(ctypes.c_double)]),
+        "mf_get_factors": (i32, [vp, vp, vp, i32]),
+        "mf_set_factors": (i32, [vp, vp, vp, i32]),
+        "mf_set_epoch": (i32, [vp, i32]),
+        "mf_get_epoch": (i32, [vp, ctypes.POINTER(i32)]),
+        "mf_export_schedule": (i32, [vp, i32, i32, vp, ctypes.POINTER(i64)]),
+        "mf_get_stats": (i32, [vp, ctypes.POINTER(Stats)]),
+        "mf_strata_holders": (i32, [u64, i32, i32, i32, i32, vp]),
+        "mf_destroy": (None, [vp]),
+        "mf_last_error": (ctypes.c_char_p, [vp]),
+        "mf_status_string": (ctypes.c_char_p, [i32]),
+    }
+    for name, (res, args) in sig.items():
+        fn = getattr(L, name)
+        fn.restype = res
+        fn.argtypes = args
+    _lib = L
+    return L
+
+
+def strata_holders(seed: int, a: int, world: int, t: int, j: int) -> list[int]:
+    """Host-only planner: rank holding each Q segment in sub-epoch j of epoch t."""
+    out = (ctypes.c_int32 * a)()
+    st = lib().mf_strata_holders(seed, a, world, t, j, out)
+    if st != 0:
+        raise MFError(st, "mf_strata_holders")
+    return list(out)
+
+
+def _torch():
+    import torch
+    return torch
+
+
+class _TorchAllocator:
+    """mf_allocator hooks backed by torch's CUDA caching allocator."""
+
+    def __init__(self, device: int):
+        torch = _torch()
+        self.device = device
+        self.sizes = {}
+
+        def _alloc(nbytes, stream, user):
+            try:
+                ptr = torch.cuda.caching_allocator_alloc(int(nbytes), device, int(stream or 0))
+                return ptr
+            except Exception:  # OOM -> NULL -> MF_E_NOMEM
+                return None
+
+        def _free(ptr, nbytes, stream, user):
+            if ptr:
+                torch.cuda.caching_allocator_delete(ptr)
+
+        self._a = _ALLOC_FN(_alloc)
+        self._f = _FREE_FN(_free)
+        self.struct = Allocator(self._a, self._f, None)
+
+
+def _as_ptr(x, dtype, on_device: bool):
+    """(pointer, keepalive) for a numpy array or torch tensor of the given dtype."""
+    if on_device:
+        torch = _torch()
+        t = x if isinstance(x, torch.Tensor) else torch.as_tensor(x)
+        want = {np.int32: torch.int32, np.float32: torch.float32}[dtype]
+        t = t.to(dtype=want).contiguous()
+        return ctypes.c_void_p(t.data_ptr()), t
+    a = np.ascontiguousarray(x, dtype=dtype)
+    return ctypes.c_void_p(a.ctypes.data), a
+
+
+class MF:
+    """One training context (one GPU / one rank).  Mirrors include/mf.h."""
+
+    def __init__(self, m: int, n: int, k: int = 128, *, lambda_p: float = 0.05,
+                 lambda_q: float | None = None, alpha: float = 0.08, beta: float = 0.3,
+                 init_scale: float = 1.0, rating_scale: float = 1.0, seed: int = 42,
+                 schedule: str = "hogwild", storage: str = "fp32", workers: int = 0,
+                 batch_f: int = 256, wf_cols: int = 0, grid_a: int = 0, cyclic: bool = False,
+                 lane_bytes: int = 0, device: int = 0, rank: int = 0, world: int = 1,
+                 nccl_id: bytes | None = None, stream=None, allocator: str = "torch"):
+        L = lib()
+        p = Params()
+        L.mf_params_default(ctypes.byref(p))
+        p.m, p.n, p.k = int(m), int(n), int(k)
+        p.lambda_p = lambda_p
+        p.lambda_q = lambda_p if lambda_q is None else lambda_q
+        p.alpha, p.beta, p.init_scale, p.rating_scale = alpha, beta, init_scale, rating_scale
+        p.seed = seed
+        p.schedule, p.storage = SCHEDULE[schedule], STORAGE[storage]
+        p.workers, p.batch_f, p.wf_cols, p.grid_a = workers, batch_f, wf_cols, grid_a
+        p.cyclic, p.lane_bytes = int(cyclic), lane_bytes
+        p.device, p.rank, p.world = device, rank, world
+        self._id_buf = None
+        if nccl_id is not None:
+            self._id_buf = ctypes.create_string_buffer(bytes(nccl_id), 128)
+            p.nccl_id = ctypes.cast(self._id_buf, ctypes.c_void_p)
+        torch = _torch()
+        if stream is None and torch.cuda.is_available():
+            stream = torch.cuda.current_stream(device)
+        if stream is not None:
+            p.stream = ctypes.c_void_p(int(getattr(stream, "cuda_stream", stream)) or None)
+        self._alloc = None
+        if allocator == "torch" and torch.cuda.is_available():
+            self._alloc = _TorchAllocator(device)
+            p.alloc = ctypes.pointer(self._alloc.struct)
+        self.params = p
+        self.m, self.n, self.k = int(m), int(n), int(k)
+        self.device = device
+        h = ctypes.c_void_p()
+        st = L.mf_create(ctypes.byref(p), ctypes.byref(h))
+        if st != 0:
+            raise MFError(st, "mf_create")
+        self.h = h
+
+    # -- helpers
+    def _check(self, st: int, what: str):
+        if st != 0:
+            msg = lib().mf_last_error(self.h)
+            raise MFError(st, f"{what}: {msg.decode() if msg else ''}")
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().mf_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    # -- API
+    def load(self, u, v, r, set: str = "train", on_device: bool | None = None):
+        if on_device is None:
+            on_device = _is_cuda_tensor(u)
+        pu, ku = _as_ptr(u, np.int32, on_device)
+        pv, kv = _as_ptr(v, np.int32, on_device)
+        pr, kr = _as_ptr(r, np.float32, on_device)
+        n = len(ku)
+        self._check(lib().mf_load_coo(self.h, SETS[set], n, pu, pv, pr, int(on_device)),
+                    f"mf_load_coo({set})")
+
+    def train_epoch(self) -> int:
+        t = ctypes.c_int32(0)
+        self._check(lib().mf_train_epoch(self.h, ctypes.byref(t)), "mf_train_epoch")
+        return t.value
+
+    def rmse(self, set: str = "test") -> float:
+        out = ctypes.c_double(0)
+        self._check(lib().mf_rmse(self.h, SETS[set], ctypes.byref(out)), "mf_rmse")
+        return out.value
+
+    def factors(self, on_device: bool = False):
+        if on_device:
+            torch = _torch()
+            P = torch.empty((self.m, self.k), dtype=torch.float32, device=f"cuda:{self.device}")
+            Q = torch.empty((self.n, self.k), dtype=torch.float32, device=f"cuda:{self.device}")
+            self._check(lib().mf_get_factors(self.h, ctypes.c_void_p(P.data_ptr()),
+                                             ctypes.c_void_p(Q.data_ptr()), 1), "mf_get_factors")
+            return P, Q
+        P = np.empty((self.m, self.k), dtype=np.float32)
+        Q = np.empty((self.n, self.k), dtype=np.float32)
+        self._check(lib().mf_get_factors(self.h, P.ctypes.data, Q.ctypes.data, 0), "mf_get_factors")
+        return P, Q
+
+    def set_factors(self, P=None, Q=None):
+        P = None if P is None else np.ascontiguousarray(P, dtype=np.float32)
+        Q = None if Q is None else np.ascontiguousarray(Q, dtype=np.float32)
+        self._check(lib().mf_set_factors(self.h, None if P is None else P.ctypes.data,
+                                         None if Q is None else Q.ctypes.data, 0), "mf_set_factors")
+
+    @property
+    def epoch(self) -> int:
+        t = ctypes.c_int32(0)
+        self._check(lib().mf_get_epoch(self.h, ctypes.byref(t)), "mf_get_epoch")
+        return t.value
+
+    def set_epoch(self, t: int):
+        self._check(lib().mf_set_epoch(self.h, t), "mf_set_epoch")
+
+    def export(self, what: str, epoch: int = 0) -> np.ndarray:
+        n = ctypes.c_int64(0)
+        self._check(lib().mf_export_schedule(self.h, EXPORTS[what], epoch, None, ctypes.byref(n)),
+                    f"export({what})")
+        buf = np.empty(max(n.value, 1), dtype=np.int64)
+        self._check(lib().mf_export_schedule(self.h, EXPORTS[what], epoch, buf.ctypes.data,
+                                             ctypes.byref(n)), f"export({what})")
+        return buf[:n.value]
+
+    def stats(self) -> dict:
+        s = Stats()
+        self._check(lib().mf_get_stats(self.h, ctypes.byref(s)), "mf_get_stats")
+        return {name: getattr(s, name) for name, _ in Stats._fields_}
+
+
+def _is_cuda_tensor(x) -> bool:
+    try:
+        import torch
+        return isinstance(x, torch.Tensor) and x.is_cuda
+    except ImportError:
+        return False
+
+
+def nccl_unique_id_via(group=None) -> bytes:
+    """Create an ncclUniqueId on rank 0 and broadcast it over torch.distributed (gloo or nccl)."""
+    torch = _torch()
+    import torch.distributed as dist
+    if dist.get_rank(group) == 0:
+        uid = _nccl_get_unique_id()
+        t = torch.tensor(list(uid), dtype=torch.uint8)
+    else:
+        t = torch.zeros(128, dtype=torch.uint8)
+    if dist.get_backend(group) == "nccl":
+        t = t.cuda()
+    dist.broadcast(t, src=0, group=group)
+    return bytes(t.cpu().tolist())
+
+
+def _nccl_get_unique_id() -> bytes:
+    for name in ("libnccl.so.2", "libnccl.so"):
+        try:
+            L = ctypes.CDLL(name, mode=ctypes.RTLD_GLOBAL)
+            break
+        except OSError:
+            L = None
+    if L is None:
+        raise MFError(-4, "libnccl.so.2 not loadable")
+    buf = ctypes.create_string_buffer(128)
+    st = L.ncclGetUniqueId(buf)
+    if st != 0:
+        raise MFError(-4, f"ncclGetUniqueId -> {st}")
+    return buf.raw

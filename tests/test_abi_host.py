@@ -1,0 +1,83 @@
+"""C-ABI library checks that need no GPU: it loads, exports every symbol include/mf.h declares,
+and its host-only logic (parameter defaults, strata planner) is right."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+from paper_conf_hpdc_xietfl17_b200 import build, mf
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def L():
+    build.build()
+    return mf.lib()
+
+
+def declared_symbols():
+    src = open(os.path.join(ROOT, "include", "mf.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(mf_[a-z_]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol(L):
+    names = declared_symbols()
+    assert "mf_train_epoch" in names and "mf_create" in names and len(names) >= 15
+    for name in names:
+        assert hasattr(L, name), name
+    assert set(names) <= set(mf.EXPORTED)
+
+
+def test_abi_version_and_status_strings(L):
+    assert L.mf_abi_version() == 1
+    assert L.mf_status_string(-6) == b"MF_E_RANGE"
+
+
+def test_params_default_and_struct_size(L):
+    p = mf.Params()
+    assert L.mf_params_default(ctypes.byref(p)) == 0
+    assert p.struct_size == ctypes.sizeof(mf.Params)
+    # Table 3 Netflix and Table 2 k
+    assert (p.k, round(p.lambda_p, 6), round(p.alpha, 6), round(p.beta, 6)) == (128, 0.05, 0.08, 0.3)
+    assert p.batch_f == 256 and p.world == 1
+
+
+def test_create_rejects_bad_params_before_touching_a_device(L):
+    p = mf.Params()
+    L.mf_params_default(ctypes.byref(p))
+    h = ctypes.c_void_p()
+    p.m, p.n = 100, 100
+    p.k = 48
+    assert L.mf_create(ctypes.byref(p), ctypes.byref(h)) == -7      # k not supported
+    p.k = 16
+    p.storage = 5
+    assert L.mf_create(ctypes.byref(p), ctypes.byref(h)) == -1
+    p.storage = 0
+    p.world, p.grid_a = 3, 8                                         # a % world != 0
+    assert L.mf_create(ctypes.byref(p), ctypes.byref(h)) == -1
+    bad = mf.Params()
+    assert L.mf_create(ctypes.byref(bad), ctypes.byref(h)) == -1     # struct_size unset
+    assert not h.value
+
+
+def test_strata_holders_partition_and_rotation(L):
+    """A: in sub-epoch j segment J is held by the owner of row (J - pi_t[j]) mod a; each rank
+    holds exactly a/G segments per sub-epoch; pi_t is the oracle's strata order."""
+    from oracle import pyoracle as po
+    a = 8
+    for G in (1, 2, 4, 8):
+        for t in range(3):
+            o = po.Oracle(16, 16, 2, [0], [0], [1.0], seed=42, grid_a=a)
+            pi = o.export("strata", t)
+            for j in range(a):
+                h = mf.strata_holders(42, a, G, t, j)
+                assert sorted(np.bincount(h, minlength=G).tolist()) == [a // G] * G
+                for J in range(a):
+                    r = (J - pi[j]) % a
+                    assert h[J] == r // (a // G)
+    with pytest.raises(mf.MFError):
+        mf.strata_holders(42, 8, 3, 0, 0)
