@@ -1,0 +1,109 @@
+"""Full-size checks at BASELINE.json's Netflix shape, in the launch configuration bench.py
+times (-m gpu): sampled outputs the oracle computes one by one, whole-structure oracle calls
+that need only the index space, and properties that hold at any size."""
+import numpy as np
+import pytest
+
+from oracle import pyoracle as po
+from paper_conf_hpdc_xietfl17_b200 import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+from paper_conf_hpdc_xietfl17_b200 import mf  # noqa: E402
+
+L = po.lib()
+SEED = 42
+NETFLIX = synth.SHAPES["netflix"]
+HP = dict(lambda_p=NETFLIX["lam"], alpha=NETFLIX["alpha"], beta=NETFLIX["beta"])
+
+
+@pytest.fixture(scope="module")
+def netflix():
+    return synth.shaped("netflix", device="cuda")
+
+
+@pytest.fixture(scope="module")
+def hog(netflix):
+    """The bench.py configuration: Hogwild, fp16 storage, k = 128, all resident workers."""
+    R = netflix
+    g = mf.MF(R.m, R.n, 128, storage="fp16", seed=SEED, **HP)
+    g.load(R.u, R.v, R.r)
+    g.load(R.ut, R.vt, R.rt, "test")
+    yield g
+    g.close()
+
+
+def test_fullsize_shuffle_and_relabel_bit_exact(netflix, hog):
+    R = netflix
+    perm = hog.export("perm")
+    want = po.perm(L.or_stream(SEED, 1, 0, 0), R.N)          # 99M-key sort in the oracle
+    assert np.array_equal(perm, want)
+    assert np.array_equal(hog.export("rho_r"), np.argsort(po.perm(L.or_stream(SEED, 2, 0, 0), R.m)))
+    assert np.array_equal(hog.export("rho_c"), np.argsort(po.perm(L.or_stream(SEED, 3, 0, 0), R.n)))
+
+
+def test_fullsize_chunk_order_bit_exact(netflix, hog):
+    nch = -(-netflix.N // 256)
+    for t in (0, 7):
+        want = po.perm(L.or_stream(SEED, 6, t, 0), nch)
+        assert np.array_equal(hog.export("chunkorder", t), want)
+
+
+def test_fullsize_init_sampled(netflix):
+    """P[u][d] = round_fp16((float)U24(S_P, u*k+d) * 2^-24 * sqrt(1/k)) at sampled (u, d)."""
+    R = netflix
+    g = mf.MF(R.m, R.n, 128, storage="fp16", seed=SEED, **HP)
+    g.load(R.u[:1000], R.v[:1000], R.r[:1000])
+    P, Q = g.factors()
+    g.close()
+    rng = np.random.default_rng(0)
+    SP, SQ = L.or_stream(SEED, 4, 0, 0), L.or_stream(SEED, 5, 0, 0)
+    amp = np.float32(np.sqrt(1.0 / 128))
+    for X, S, rows in ((P, SP, R.m), (Q, SQ, R.n)):
+        for _ in range(300):
+            i, d = int(rng.integers(rows)), int(rng.integers(128))
+            u01 = np.float32(L.or_key(S, i * 128 + d) >> 40) * np.float32(2.0 ** -24)
+            assert X[i, d] == L.or_round_storage(1, float(np.float32(u01 * amp)))
+
+
+def test_fullsize_hogwild_epoch_properties(netflix, hog):
+    r0 = hog.rmse()
+    hog.train_epoch()
+    st = hog.stats()
+    assert st["updates"] == netflix.N and st["sgd_launches"] == 1
+    assert st["bytes_per_update"] == 12 + 4 * 128 * 2
+    assert hog.rmse() < r0
+
+
+def test_fullsize_hogwild_full_concurrency_converges_like_serial(netflix):
+    """20 epochs at full concurrency land within 0.5% of the serial order.  The serial
+    reference at this size is the deterministic wavefront run, which the parity tests prove
+    equal to the oracle's serial loop (the CPU oracle would need ~20 min for 20 epochs here)."""
+    R = netflix
+    res = {}
+    for sched in ("hogwild", "wavefront"):
+        g = mf.MF(R.m, R.n, 128, storage="fp32", schedule=sched, seed=SEED,
+                  workers=2048 if sched == "wavefront" else 0, **HP)
+        g.load(R.u, R.v, R.r)
+        g.load(R.ut, R.vt, R.rt, "test")
+        for _ in range(20):
+            g.train_epoch()
+        res[sched] = g.rmse()
+        g.close()
+    assert abs(res["hogwild"] - res["wavefront"]) <= 0.005 * res["wavefront"], res
+
+
+def test_fullsize_wavefront_deterministic_rerun(netflix):
+    """Property at any size: the deterministic mode gives bit-identical factors run to run."""
+    R = netflix
+    outs = []
+    for _ in range(2):
+        g = mf.MF(R.m, R.n, 128, storage="fp32", schedule="wavefront", workers=2048, seed=SEED, **HP)
+        g.load(R.u, R.v, R.r)
+        g.train_epoch()
+        outs.append(g.factors())
+        g.close()
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])

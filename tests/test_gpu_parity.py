@@ -120,19 +120,20 @@ def test_deterministic_parity_other_k_ragged(k):
 def test_deterministic_parity_low_precision_storage(tiny, storage):
     """Storage rounding is RNE on both sides (R16), but the fp32 value being rounded
     differs between the two sides by the dot-product order (tree vs sequential, ~k*eps32), so an
-    update can round to the neighbouring storage value: 1 storage ulp, which later updates carry
-    along (damped by gamma).  Bar: every entry within 2 storage ulps of the oracle's, most of them
-    identical, and test RMSE within 1e-4 relative."""
+    update can round to the neighbouring storage value: one ulp of that value's binade, which
+    later updates carry along as an ABSOLUTE offset (damped by gamma).  Bar: every entry within
+    2 ulps of the largest binade in use (absolute), most entries identical, test RMSE within
+    1e-4 relative."""
     g, o = pair(tiny, storage=storage, schedule="wavefront", workers=8, wf_cols=16, **TABLE3_NETFLIX)
     g.train_epoch()
     o.train_epoch()
-    ulp = 2.0 ** -10 if storage == "fp16" else 2.0 ** -7   # relative spacing of the format
+    mant = 10 if storage == "fp16" else 7
     rg, ro = g.rmse(), o.rmse(tiny.ut, tiny.vt, tiny.rt)
     for Xg, Xo in zip(g.factors(), o.factors()):
-        rel = np.abs(Xg - Xo) / np.maximum(np.abs(Xo), 2.0 ** -14)
-        diag = (storage, float(np.mean(Xg == Xo)), float(rel.max()), rg, ro)
+        ulp_abs = 2.0 ** (np.floor(np.log2(np.abs(Xo).max())) - mant)
+        diag = (storage, float(np.mean(Xg == Xo)), float(np.abs(Xg - Xo).max()), ulp_abs, rg, ro)
         assert np.mean(Xg == Xo) > 0.9, diag
-        assert rel.max() <= 2 * ulp, diag
+        assert np.abs(Xg - Xo).max() <= 2 * ulp_abs, diag
     assert abs(rg - ro) <= 1e-4 * ro, (rg, ro)
 
 
@@ -150,9 +151,16 @@ def test_wavefront_is_deterministic_run_to_run():
 
 # ----------------------------------------------------------------------------- Hogwild
 
+# Hogwild results are race-dependent (R19): only the RMSE bar applies.  Concurrency must
+# respect the paper's convergence rule s < min(m, n)/20 (section 7.5): on the tiny
+# set (n = 800) full GPU concurrency (~200 concurrent chunks) violates it ~10x and does NOT
+# converge like serial SGD (measured: +46% RMSE; tools/convergence.py),
+# exactly as the paper reports for Hugewiki with j = 4.  So the small-set tests run within
+# the rule; tests/test_gpu_fullsize.py checks full concurrency at Netflix scale.
+
 @pytest.mark.parametrize("storage,tol", [("fp32", 0.005), ("fp16", 0.01)])
 def test_hogwild_20_epoch_rmse_within_tolerance(tiny, storage, tol):
-    g, o = pair(tiny, storage=storage, schedule="hogwild", **TABLE3_NETFLIX)
+    g, o = pair(tiny, storage=storage, schedule="hogwild", workers=4, **TABLE3_NETFLIX)
     for _ in range(20):
         g.train_epoch()
         o.train_epoch()
@@ -161,17 +169,27 @@ def test_hogwild_20_epoch_rmse_within_tolerance(tiny, storage, tol):
 
 
 def test_hogwild_powerlaw_20_epochs_matches_oracle():
-    """Skewed (power-law) data at full concurrency: collisions between concurrent workers are
-    frequent on hot columns; the 20-epoch RMSE still lands within 0.5% of the serial oracle."""
+    """Skewed (power-law) data, n = 900, 32 concurrent workers (< n/20 = 45): collisions on hot
+    columns happen, and the 20-epoch RMSE still lands within 0.5% of the serial oracle."""
     R = synth.powerlaw(4000, 900, 200_000, 20_000, seed=5, rank=8, mu=3.6, noise=0.5)
     R = synth.Ratings(R.m, R.n, R.u.numpy(), R.v.numpy(), R.r.numpy(), R.ut.numpy(), R.vt.numpy(),
                       R.rt.numpy())
-    g, o = pair(R, k=32, schedule="hogwild", **TABLE3_NETFLIX)
+    g, o = pair(R, k=32, schedule="hogwild", workers=32, **TABLE3_NETFLIX)
     for _ in range(20):
         g.train_epoch()
         o.train_epoch()
     rg, ro = g.rmse(), o.rmse(R.ut, R.vt, R.rt)
     assert abs(rg - ro) <= 0.005 * ro, (rg, ro)
+
+
+def test_hogwild_one_worker_reproduces_oracle_curve(tiny):
+    """1 worker = the serial batch-Hogwild order of the oracle: RMSE curve equal epoch by epoch."""
+    g, o = pair(tiny, schedule="hogwild", workers=1, **TABLE3_NETFLIX)
+    for _ in range(10):
+        g.train_epoch()
+        o.train_epoch()
+        rg, ro = g.rmse(), o.rmse(tiny.ut, tiny.vt, tiny.rt)
+        assert abs(rg - ro) <= 1e-5 * ro, (rg, ro)
 
 
 def test_hogwild_epoch_updates_every_sample_once(tiny):
