@@ -118,6 +118,22 @@ __global__ void k_histogram(const uint32_t* __restrict__ bucket, int64_t N,
     atomicAdd(cnt + bucket[j], 1u);
 }
 
+// Few buckets (strata blocks, a*a <= 4096): per-CTA shared-memory counts, one global atomic
+// per bucket per CTA (a single global counter would serialise N atomics).
+constexpr int kSmemBuckets = 4096;
+__global__ void k_histogram_smem(const uint32_t* __restrict__ bucket, int64_t N, int nb,
+                                 unsigned int* __restrict__ cnt) {
+  __shared__ unsigned int h[kSmemBuckets];
+  for (int i = threadIdx.x; i < nb; i += blockDim.x) h[i] = 0u;
+  __syncthreads();
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < N;
+       j += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(h + bucket[j], 1u);
+  __syncthreads();
+  for (int i = threadIdx.x; i < nb; i += blockDim.x)
+    if (h[i]) atomicAdd(cnt + i, h[i]);
+}
+
 // Place sorted sample x (bucket b = key[x]) at slot dst_off[b] + (x - src_off[b]).
 __global__ void k_place(const uint32_t* __restrict__ keys_sorted,
                         const uint32_t* __restrict__ pos_sorted, int64_t N,
@@ -791,7 +807,10 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
   TRY(c->alloc(&cnt, (size_t)nbuckets));
   CUDA_TRY(c, cudaMemsetAsync(cnt, 0, nbuckets * 4, c->st));
   if (N > 0) {
-    k_histogram<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(bk0, N, cnt);
+    if (nbuckets <= kSmemBuckets)
+      k_histogram_smem<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(bk0, N, (int)nbuckets, cnt);
+    else
+      k_histogram<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(bk0, N, cnt);
     KERNEL_TRY(c);
   }
   // stable sort of storage positions by bucket (radix sort is stable; storage order kept, R12)

@@ -21,6 +21,7 @@ __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slot
                                                  int workers, T* __restrict__ P, T* __restrict__ Q,
                                                  int f, float g, float lp, float lq) {
   constexpr int GPW = 32 / L;
+  const float cp = 1.f - g * lp, cq = 1.f - g * lq;
   const int lane = threadIdx.x & 31;
   const int grp = lane / L, gl = lane % L, gbase = grp * L;
   const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
@@ -43,7 +44,7 @@ __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slot
       lo = (int64_t)chunk * f;
       hi = lo + f;
     }
-    run_serial<T, K, L>(slots, lo, hi, P, Q, g, lp, lq, gl, gbase, gmask);
+    run_serial<T, K, L>(slots, lo, hi, P, Q, g, cp, cq, gl, gbase, gmask);
   }
 }
 
@@ -77,6 +78,7 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
   const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
   const int worker = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) / L);
   if (worker >= s) return;
+  const float cp = 1.f - g * lp, cq = 1.f - g * lq;
   const int32_t* my_seq = seq + (int64_t)worker * c;
   const int32_t* my_rank = rank + (int64_t)worker * c;
   for (int w = 0; w < c; ++w) {
@@ -84,7 +86,7 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
     const int tgt = __ldg(my_rank + w);
     while (ld_acquire(tickets + col) != tgt) __nanosleep(64);
     const int64_t sb = (int64_t)worker * c + col;
-    run_serial<T, K, L>(slots, __ldg(sub_off + sb), __ldg(sub_off + sb + 1), P, Q, g, lp, lq, gl,
+    run_serial<T, K, L>(slots, __ldg(sub_off + sb), __ldg(sub_off + sb + 1), P, Q, g, cp, cq, gl,
                         gbase, gmask);
     __threadfence();
     __syncwarp(gmask);
