@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--wf-cols", type=int, default=0)
     ap.add_argument("--cyclic", action="store_true")
     ap.add_argument("--lane-bytes", type=int, default=0)
+    ap.add_argument("--prefetch", type=int, default=0)
     ap.add_argument("--fraction", type=float, default=1.0, help="scale the workload (testing)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -226,7 +227,7 @@ def main():
     if world > 1:
         nccl_id = mf.nccl_unique_id_via()
     kw = dict(schedule=args.schedule, storage=args.storage, workers=args.workers,
-              wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes, seed=42,
+              wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes, prefetch=args.prefetch, seed=42,
               device=local, rank=rank, world=world, nccl_id=nccl_id, **hp)
     torch.cuda.synchronize()
     model = mf.MF(R.m, R.n, args.k, stream=stream, **kw)

@@ -85,6 +85,7 @@ typedef struct mf_params {
   int32_t grid_a;         /* strata grid a x a (0 = 1 if world == 1 else 8); a % world == 0      */
   int32_t cyclic;         /* wavefront: 1 = cyclic column order (A: cyclic variant), needs c >= s */
   int32_t lane_bytes;     /* Hogwild/RMSE kernel: bytes of p_u (and q_v) per lane, 16 or 32 (0 = 16) */
+  int32_t prefetch;       /* Hogwild software-pipeline depth: samples in flight per worker, 1 or 2 (0 = 1) */
   int32_t device;         /* CUDA device ordinal                                                */
   int32_t rank, world;    /* world > 1: DSGD strata over `world` GPUs, one ctx per rank         */
   int32_t transport;      /* 0 = NCCL (world > 1)                                              */

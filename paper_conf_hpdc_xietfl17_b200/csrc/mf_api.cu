@@ -553,6 +553,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
     return MF_E_INVAL;
   if (!(p->rating_scale > 0.f) || !(p->init_scale > 0.f)) return MF_E_INVAL;
   if (p->lane_bytes != 0 && p->lane_bytes != 16 && p->lane_bytes != 32) return MF_E_INVAL;
+  if (p->prefetch < 0 || p->prefetch > 2) return MF_E_INVAL;
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
   const int a = p->grid_a > 0 ? p->grid_a : (world == 1 ? 1 : 8);
@@ -1034,6 +1035,7 @@ static mf_status run_stratum(mf_ctx* c, int32_t t, int j, const std::vector<int6
     CUDA_TRY(c, cudaMemsetAsync(c->counter, 0, sizeof(unsigned long long), c->st));
     HogwildLaunch L{};
     L.storage = c->p.storage; L.k = c->k; L.lane_bytes = c->p.lane_bytes ? c->p.lane_bytes : 16;
+    L.prefetch = c->p.prefetch ? c->p.prefetch : 1;
     L.slots = c->slots; L.chunks = c->chunk_order; L.segs = segs; L.counter = c->counter;
     L.workers = c->p.workers; L.num_sms = c->num_sms; L.f = c->f;
     L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;

@@ -19,7 +19,7 @@ struct ChunkSegs {
 };
 
 struct HogwildLaunch {
-  int storage, k, lane_bytes;
+  int storage, k, lane_bytes, prefetch;
   const Rating* slots;
   const uint32_t* chunks;
   ChunkSegs segs;

@@ -14,7 +14,7 @@ namespace mfb {
 // f consecutive slots of its chunk serially.  Persistent grid: workers loop until the list is
 // exhausted.  The chunk list of a launch is the concatenation of up to kMaxSegs block segments.
 // ---------------------------------------------------------------------------------------------
-template <typename T, int K, int L>
+template <typename T, int K, int L, int D>
 __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slots,
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
                                                  unsigned long long* __restrict__ counter,
@@ -24,7 +24,6 @@ __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slot
   const float cp = 1.f - g * lp, cq = 1.f - g * lq;
   const int lane = threadIdx.x & 31;
   const int grp = lane / L, gl = lane % L, gbase = grp * L;
-  const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
   const int warp = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) >> 5);
   const int first = warp * GPW;
   if (first >= workers) return;                      // warp-uniform
@@ -36,15 +35,16 @@ __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slot
     base = __shfl_sync(0xffffffffu, base, 0);
     if ((int64_t)base >= total) break;
     const int64_t ci = (int64_t)base + grp;
-    int64_t lo = 0, hi = 0;
-    if (grp < nact && ci < total) {
+    const bool act = grp < nact && ci < total;
+    int64_t lo = 0;
+    if (act) {
       int sgi = 0;
       while (ci >= segs.prefix[sgi + 1]) ++sgi;
       const uint32_t chunk = __ldg(chunks + segs.begin[sgi] + (ci - segs.prefix[sgi]));
       lo = (int64_t)chunk * f;
-      hi = lo + f;
     }
-    run_serial<T, K, L>(slots, lo, hi, P, Q, g, cp, cq, gl, gbase, gmask);
+    // every group of the warp runs f iterations in lockstep (inactive ones on sentinels)
+    run_serial<T, K, L, D, true>(slots, lo, f, act, P, Q, g, cp, cq, gl, gbase, 0xffffffffu);
   }
 }
 
@@ -86,8 +86,9 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
     const int tgt = __ldg(my_rank + w);
     while (ld_acquire(tickets + col) != tgt) __nanosleep(64);
     const int64_t sb = (int64_t)worker * c + col;
-    run_serial<T, K, L>(slots, __ldg(sub_off + sb), __ldg(sub_off + sb + 1), P, Q, g, cp, cq, gl,
-                        gbase, gmask);
+    const int64_t lo = __ldg(sub_off + sb);
+    run_serial<T, K, L, 2, false>(slots, lo, (int)(__ldg(sub_off + sb + 1) - lo), true, P, Q, g, cp,
+                                  cq, gl, gbase, gmask);
     __threadfence();
     __syncwarp(gmask);
     if (gl == 0) st_release(tickets + col, tgt + 1);
@@ -161,9 +162,9 @@ __global__ void k_rmse_final(const double* __restrict__ partial, int n, double* 
 // ---------------------------------------------------------------------------------------------
 // Dispatch
 // ---------------------------------------------------------------------------------------------
-template <typename T, int K, int L>
+template <typename T, int K, int L, int D>
 static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
-  auto kern = k_hogwild<T, K, L>;
+  auto kern = k_hogwild<T, K, L, D>;
   const int threads = 256;
   int per_sm = 0;
   cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, 0);
@@ -225,11 +226,16 @@ static constexpr int lanes_for(int K, int S, int LB) {
   return (K * S / LB) >= 32 ? 32 : ((K * S / LB) < 1 ? 1 : (K * S / LB));
 }
 
+template <typename T, int K, int LB>
+static cudaError_t hogwild_kl(const HogwildLaunch& a) {
+  constexpr int S = (int)sizeof(T);
+  if (a.prefetch == 1) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1>(a);
+  return launch_hogwild_t<T, K, lanes_for(K, S, LB), 2>(a);
+}
 template <typename T, int K>
 static cudaError_t hogwild_k(const HogwildLaunch& a) {
-  constexpr int S = (int)sizeof(T);
-  if (a.lane_bytes == 32) return launch_hogwild_t<T, K, lanes_for(K, S, 32)>(a);
-  return launch_hogwild_t<T, K, lanes_for(K, S, 16)>(a);
+  if (a.lane_bytes == 32) return hogwild_kl<T, K, 32>(a);
+  return hogwild_kl<T, K, 16>(a);
 }
 template <typename T, int K>
 static cudaError_t rmse_k(const RmseLaunch& a) {

@@ -47,7 +47,8 @@ class Params(ctypes.Structure):
                 ("storage", ctypes.c_int32), ("workers", ctypes.c_int32),
                 ("batch_f", ctypes.c_int32), ("wf_cols", ctypes.c_int32),
                 ("grid_a", ctypes.c_int32), ("cyclic", ctypes.c_int32),
-                ("lane_bytes", ctypes.c_int32), ("device", ctypes.c_int32),
+                ("lane_bytes", ctypes.c_int32), ("prefetch", ctypes.c_int32),
+                ("device", ctypes.c_int32),
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("transport", ctypes.c_int32), ("nccl_id", ctypes.c_void_p),
                 ("stream", ctypes.c_void_p), ("alloc", ctypes.POINTER(Allocator))]
@@ -163,7 +164,7 @@ class MF:
                  init_scale: float = 1.0, rating_scale: float = 1.0, seed: int = 42,
                  schedule: str = "hogwild", storage: str = "fp32", workers: int = 0,
                  batch_f: int = 256, wf_cols: int = 0, grid_a: int = 0, cyclic: bool = False,
-                 lane_bytes: int = 0, device: int = 0, rank: int = 0, world: int = 1,
+                 lane_bytes: int = 0, prefetch: int = 0, device: int = 0, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, stream=None, allocator: str = "torch"):
         L = lib()
         p = Params()
@@ -175,7 +176,7 @@ class MF:
         p.seed = seed
         p.schedule, p.storage = SCHEDULE[schedule], STORAGE[storage]
         p.workers, p.batch_f, p.wf_cols, p.grid_a = workers, batch_f, wf_cols, grid_a
-        p.cyclic, p.lane_bytes = int(cyclic), lane_bytes
+        p.cyclic, p.lane_bytes, p.prefetch = int(cyclic), lane_bytes, prefetch
         p.device, p.rank, p.world = device, rank, world
         self._id_buf = None
         if nccl_id is not None:
