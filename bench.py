@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--cyclic", action="store_true")
     ap.add_argument("--lane-bytes", type=int, default=0)
     ap.add_argument("--prefetch", type=int, default=0)
+    ap.add_argument("--wf-kernel", type=int, default=0)
     ap.add_argument("--fraction", type=float, default=1.0, help="scale the workload (testing)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -227,7 +228,8 @@ def main():
     if world > 1:
         nccl_id = mf.nccl_unique_id_via()
     kw = dict(schedule=args.schedule, storage=args.storage, workers=args.workers,
-              wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes, prefetch=args.prefetch, seed=42,
+              wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes, prefetch=args.prefetch,
+              wf_kernel=args.wf_kernel, seed=42,
               device=local, rank=rank, world=world, nccl_id=nccl_id, **hp)
     torch.cuda.synchronize()
     model = mf.MF(R.m, R.n, args.k, stream=stream, **kw)

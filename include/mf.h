@@ -79,13 +79,15 @@ typedef struct mf_params {
   int32_t schedule;       /* mf_schedule                                                        */
   int32_t storage;        /* mf_storage of P and Q; arithmetic is always fp32                   */
   int32_t workers;        /* s: Hogwild = concurrent sample groups (0 = all resident);
-                             wavefront = row sub-blocks per strata block (0 = 2048)             */
+                             wavefront = row sub-blocks per strata block (0 = min(1024, m/(4a)))             */
   int32_t batch_f;        /* Eq. 8 batch f (0 = 256)                                    */
   int32_t wf_cols;        /* wavefront column sub-blocks c (0 = 2*s, R9)                        */
   int32_t grid_a;         /* strata grid a x a (0 = 1 if world == 1 else 8); a % world == 0      */
   int32_t cyclic;         /* wavefront: 1 = cyclic column order (A: cyclic variant), needs c >= s */
   int32_t lane_bytes;     /* Hogwild/RMSE kernel: bytes of p_u (and q_v) per lane, 16 or 32 (0 = 16) */
   int32_t prefetch;       /* Hogwild software-pipeline depth: samples in flight per worker, 1 or 2 (0 = 1) */
+  int32_t wf_kernel;      /* wavefront kernel: 0 = auto = 1 = ring-staged (cp.async smem ring),
+                             2 = register pipeline; both give the same result                   */
   int32_t device;         /* CUDA device ordinal                                                */
   int32_t rank, world;    /* world > 1: DSGD strata over `world` GPUs, one ctx per rank         */
   int32_t transport;      /* 0 = NCCL (world > 1)                                              */

@@ -150,6 +150,25 @@ __global__ void k_place(const uint32_t* __restrict__ keys_sorted,
   }
 }
 
+// Ring-staged wavefront metadata: for slot x, the distance to the previous slot of the same
+// sub-block with the same u (low byte) / same v (high byte) when it is <= W, else 0.
+__global__ void k_dupdist(const Rating* __restrict__ slots, int64_t N, Grid G, int W,
+                          uint16_t* __restrict__ dup) {
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < N;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const Rating a = slots[x];
+    const uint32_t b = bucket_of(G, a.u, a.v);
+    int pd = 0, qd = 0;
+    for (int d = 1; d <= W && x - d >= 0; ++d) {
+      const Rating y = slots[x - d];
+      if (bucket_of(G, y.u, y.v) != b) break;
+      if (!pd && y.u == a.u) pd = d;
+      if (!qd && y.v == a.v) qd = d;
+    }
+    dup[x] = (uint16_t)(pd | (qd << 8));
+  }
+}
+
 // Alg. 1 l.3 (R5): X[rho[id]][d] = round_S((float)U24(S, id*k+d) * 2^-24 * amp),
 // keyed by the ORIGINAL id (A: S_P / S_Q).
 template <typename T>
@@ -360,6 +379,7 @@ struct mf_ctx {
   void* P = nullptr;
   void* Q = nullptr;
   Rating* test = nullptr;
+  uint16_t* dup = nullptr;         // wavefront ring kernel: per-slot duplicate distances
   int64_t* sub_off = nullptr;      // wavefront: a*a*s*c + 1
   std::vector<int64_t> blk_off;    // a*a + 1 slot offsets (Hogwild: padded to f)
   std::vector<int64_t> blk_len;    // a*a sample counts
@@ -554,6 +574,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (!(p->rating_scale > 0.f) || !(p->init_scale > 0.f)) return MF_E_INVAL;
   if (p->lane_bytes != 0 && p->lane_bytes != 16 && p->lane_bytes != 32) return MF_E_INVAL;
   if (p->prefetch < 0 || p->prefetch > 2) return MF_E_INVAL;
+  if (p->wf_kernel < 0 || p->wf_kernel > 2) return MF_E_INVAL;
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
   const int a = p->grid_a > 0 ? p->grid_a : (world == 1 ? 1 : 8);
@@ -574,7 +595,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   c->wf = p->schedule == MF_WAVEFRONT;
   if (c->wf) {
     const int64_t rows_per_seg = p->m / a;
-    int64_t s = p->workers > 0 ? p->workers : std::min<int64_t>(2048, std::max<int64_t>(1, rows_per_seg / 4));
+    int64_t s = p->workers > 0 ? p->workers : std::min<int64_t>(1024, std::max<int64_t>(1, rows_per_seg / 4));
     c->s = (int)s;
     c->c = p->wf_cols > 0 ? p->wf_cols : 2 * c->s;
     if (p->cyclic && c->c < c->s) { delete c; return MF_E_INVAL; }
@@ -884,6 +905,13 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
   c->release(cnt); c->release(stor); c->release(bk0); c->release(bk1);
   c->release(pos0); c->release(pos1);
 
+  if (c->wf && c->p.wf_kernel != 2) {
+    TRY(c->alloc(&c->dup, (size_t)std::max<int64_t>(c->nslots, 1)));
+    if (N > 0) {
+      k_dupdist<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(c->slots, N, Gd, ring_window(), c->dup);
+      KERNEL_TRY(c);
+    }
+  }
   TRY(init_factors(c));
   TRY(alloc_schedule(c));
   CUDA_TRY(c, cudaStreamSynchronize(c->st));
@@ -1054,6 +1082,8 @@ static mf_status run_stratum(mf_ctx* c, int32_t t, int j, const std::vector<int6
     const int64_t base = b * (int64_t)c->s * c->c;
     WavefrontLaunch L{};
     L.storage = c->p.storage; L.k = c->k; L.slots = c->slots; L.sub_off = c->sub_off + base;
+    L.variant = c->p.wf_kernel == 2 ? 0 : 1;
+    L.dup = c->dup;
     L.seq = c->seq + base; L.rank = c->rank_arr + base; L.tickets = c->tickets;
     L.s = c->s; L.c = c->c; L.num_sms = c->num_sms; L.P = c->P; L.Q = c->Q; L.g = g;
     L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;

@@ -32,8 +32,10 @@ struct HogwildLaunch {
 };
 
 struct WavefrontLaunch {
-  int storage, k;
+  int storage, k, variant;  // variant 1 = ring-staged k_wavefront2 (needs dup), 0 = k_wavefront
   const Rating* slots;
+  const uint16_t* dup;     // per slot: distance to previous same-u (low byte) / same-v (high
+                           // byte) sample of the sub-block if <= ring_window(), else 0
   const int64_t* sub_off;  // s*c + 1 slot offsets of this strata block's sub-blocks
   const int32_t* seq;      // s*c
   const int32_t* rank;     // s*c
@@ -59,5 +61,6 @@ struct RmseLaunch {
 cudaError_t launch_hogwild(const HogwildLaunch& a);
 cudaError_t launch_wavefront(const WavefrontLaunch& a);
 cudaError_t launch_rmse(const RmseLaunch& a);
+int ring_window();  // W of k_wavefront2
 
 }  // namespace mfb

@@ -95,6 +95,49 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
   }
 }
 
+
+// Ring-staged wavefront (see run_subblock_ring): same schedule, tickets and result as
+// k_wavefront; the rows of each sub-block stream through a per-worker shared-memory ring.
+template <typename T, int K, int L, int RS, int F>
+__global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ slots,
+                                                    const uint16_t* __restrict__ dup,
+                                                    const int64_t* __restrict__ sub_off,
+                                                    const int32_t* __restrict__ seq,
+                                                    const int32_t* __restrict__ rank,
+                                                    int* __restrict__ tickets, int s, int c,
+                                                    T* __restrict__ P, T* __restrict__ Q, float g,
+                                                    float lp, float lq) {
+  extern __shared__ __align__(16) char smem[];
+  constexpr int ROWB = K * (int)sizeof(T);
+  const int lane = threadIdx.x & 31;
+  const int grp = lane / L, gl = lane % L, gbase = grp * L;
+  const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
+  const int local = threadIdx.x / L;
+  const int worker = blockIdx.x * (blockDim.x / L) + local;
+  if (worker >= s) return;
+  char* ring = smem + (size_t)local * RS * 2 * ROWB;
+  const float cp = 1.f - g * lp, cq = 1.f - g * lq;
+  const int32_t* my_seq = seq + (int64_t)worker * c;
+  const int32_t* my_rank = rank + (int64_t)worker * c;
+  for (int w = 0; w < c; ++w) {
+    const int col = __ldg(my_seq + w);
+    const int tgt = __ldg(my_rank + w);
+    const int64_t sb = (int64_t)worker * c + col;
+    const int64_t lo = __ldg(sub_off + sb);
+    const int n = (int)(__ldg(sub_off + sb + 1) - lo);
+    if (n > 0) {
+      while (ld_acquire(tickets + col) != tgt) __nanosleep(32);
+      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo, n, P, Q, g, cp, cq, gl, gmask, ring);
+      __threadfence();
+      __syncwarp(gmask);
+    } else {
+      // empty sub-block: still keep the column's visit order
+      while (ld_acquire(tickets + col) != tgt) __nanosleep(32);
+    }
+    if (gl == 0) st_release(tickets + col, tgt + 1);
+  }
+}
+
 // ---------------------------------------------------------------------------------------------
 // RMSE (R13): per-group fp32 dot, per-lane-0 fp64 accumulation, fixed-order block
 // reduction to one partial per CTA; k_rmse_final sums the partials in a fixed order.
@@ -208,6 +251,40 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
                                      a.stream);
 }
 
+
+constexpr int kRingSlots = 16, kRingAhead = 7;   // RS, F  ->  history window W = 8
+
+template <typename T, int K, int L>
+static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
+  auto kern = k_wavefront2<T, K, L, kRingSlots, kRingAhead>;
+  constexpr int ROWB = K * (int)sizeof(T);
+  const int threads = 32;                                    // one warp: 32/L workers
+  const int wpc = threads / L;
+  const size_t smem = (size_t)wpc * kRingSlots * 2 * ROWB;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  const int blocks = (int)cdiv64((int64_t)a.s, wpc);
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, smem);
+  if (e != cudaSuccess) return e;
+  if ((int64_t)per_sm * a.num_sms < blocks) return cudaErrorCooperativeLaunchTooLarge;
+  if (a.out_lanes) *a.out_lanes = L;
+  if (a.out_grid) *a.out_grid = blocks;
+  const Rating* slots = a.slots;
+  const uint16_t* dup = a.dup;
+  const int64_t* sub_off = a.sub_off;
+  const int32_t* seq = a.seq;
+  const int32_t* rank = a.rank;
+  int* tickets = a.tickets;
+  int s = a.s, c = a.c;
+  T* P = reinterpret_cast<T*>(a.P);
+  T* Q = reinterpret_cast<T*>(a.Q);
+  float g = a.g, lp = a.lp, lq = a.lq;
+  void* args[] = {&slots, &dup, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq};
+  return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, smem,
+                                     a.stream);
+}
+
 template <typename T, int K, int L>
 static cudaError_t launch_rmse_t(const RmseLaunch& a) {
   const int threads = 256;
@@ -245,6 +322,7 @@ static cudaError_t rmse_k(const RmseLaunch& a) {
 template <typename T, int K>
 static cudaError_t wavefront_k(const WavefrontLaunch& a) {
   constexpr int S = (int)sizeof(T);
+  if (a.variant == 1 && a.dup) return launch_wavefront2_t<T, K, lanes_for(K, S, 32)>(a);
   return launch_wavefront_t<T, K, lanes_for(K, S, 8)>(a);
 }
 
@@ -283,5 +361,6 @@ static cudaError_t wavefront_k(const WavefrontLaunch& a) {
 cudaError_t launch_hogwild(const HogwildLaunch& a) { MF_DISPATCH(hogwild_k, a) }
 cudaError_t launch_wavefront(const WavefrontLaunch& a) { MF_DISPATCH(wavefront_k, a) }
 cudaError_t launch_rmse(const RmseLaunch& a) { MF_DISPATCH(rmse_k, a) }
+int ring_window() { return kRingSlots - kRingAhead - 1; }
 
 }  // namespace mfb

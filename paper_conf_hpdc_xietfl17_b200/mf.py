@@ -48,6 +48,7 @@ class Params(ctypes.Structure):
                 ("batch_f", ctypes.c_int32), ("wf_cols", ctypes.c_int32),
                 ("grid_a", ctypes.c_int32), ("cyclic", ctypes.c_int32),
                 ("lane_bytes", ctypes.c_int32), ("prefetch", ctypes.c_int32),
+                ("wf_kernel", ctypes.c_int32),
                 ("device", ctypes.c_int32),
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("transport", ctypes.c_int32), ("nccl_id", ctypes.c_void_p),
@@ -164,7 +165,7 @@ class MF:
                  init_scale: float = 1.0, rating_scale: float = 1.0, seed: int = 42,
                  schedule: str = "hogwild", storage: str = "fp32", workers: int = 0,
                  batch_f: int = 256, wf_cols: int = 0, grid_a: int = 0, cyclic: bool = False,
-                 lane_bytes: int = 0, prefetch: int = 0, device: int = 0, rank: int = 0, world: int = 1,
+                 lane_bytes: int = 0, prefetch: int = 0, wf_kernel: int = 0, device: int = 0, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, stream=None, allocator: str = "torch"):
         L = lib()
         p = Params()
@@ -176,7 +177,7 @@ class MF:
         p.seed = seed
         p.schedule, p.storage = SCHEDULE[schedule], STORAGE[storage]
         p.workers, p.batch_f, p.wf_cols, p.grid_a = workers, batch_f, wf_cols, grid_a
-        p.cyclic, p.lane_bytes, p.prefetch = int(cyclic), lane_bytes, prefetch
+        p.cyclic, p.lane_bytes, p.prefetch, p.wf_kernel = int(cyclic), lane_bytes, prefetch, wf_kernel
         p.device, p.rank, p.world = device, rank, world
         self._id_buf = None
         if nccl_id is not None:
