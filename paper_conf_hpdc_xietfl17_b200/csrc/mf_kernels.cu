@@ -56,13 +56,33 @@ __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slot
 // serially, and releases the column with ticket+1.  Every wait is on a lexicographically
 // smaller visit, so with all workers co-resident (cooperative launch) there is no deadlock.
 // ---------------------------------------------------------------------------------------------
-__device__ __forceinline__ int ld_acquire(const int* p) {
+__device__ __forceinline__ int ld_relaxed(const int* p) {
   int v;
-  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  asm volatile("ld.relaxed.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
-__device__ __forceinline__ void st_release(int* p, int v) {
-  asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+__device__ __forceinline__ void st_relaxed(int* p, int v) {
+  asm volatile("st.relaxed.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void fence_acq_rel() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+
+// Acquire the column: spin with RELAXED loads (an ld.acquire per poll would emit an L1
+// invalidate each time and flood L2 with strong loads on the few ticket lines) and exponential
+// back-off, then one acquire fence (ld.relaxed + fence.acq_rel = acquire pattern).
+__device__ __forceinline__ void ticket_acquire(const int* t, int tgt) {
+  unsigned ns = 32;
+  while (ld_relaxed(t) != tgt) {
+    __nanosleep(ns);
+    if (ns < 1024) ns <<= 1;
+  }
+  fence_acq_rel();
+}
+// Release: every lane fences its own row stores, the group re-converges (memory ordering among
+// the participating lanes), and one lane publishes ticket+1 (fence + relaxed store = release).
+__device__ __forceinline__ void ticket_release(int* t, int next, unsigned gmask, int gl) {
+  fence_acq_rel();
+  __syncwarp(gmask);
+  if (gl == 0) st_relaxed(t, next);
 }
 
 template <typename T, int K, int L>
@@ -84,14 +104,12 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
   for (int w = 0; w < c; ++w) {
     const int col = __ldg(my_seq + w);
     const int tgt = __ldg(my_rank + w);
-    while (ld_acquire(tickets + col) != tgt) __nanosleep(64);
+    ticket_acquire(tickets + col, tgt);
     const int64_t sb = (int64_t)worker * c + col;
     const int64_t lo = __ldg(sub_off + sb);
     run_serial<T, K, L, 2, false>(slots, lo, (int)(__ldg(sub_off + sb + 1) - lo), true, P, Q, g, cp,
                                   cq, gl, gbase, gmask);
-    __threadfence();
-    __syncwarp(gmask);
-    if (gl == 0) st_release(tickets + col, tgt + 1);
+    ticket_release(tickets + col, tgt + 1, gmask, gl);
   }
 }
 
@@ -125,16 +143,9 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     const int64_t sb = (int64_t)worker * c + col;
     const int64_t lo = __ldg(sub_off + sb);
     const int n = (int)(__ldg(sub_off + sb + 1) - lo);
-    if (n > 0) {
-      while (ld_acquire(tickets + col) != tgt) __nanosleep(32);
-      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo, n, P, Q, g, cp, cq, gl, gmask, ring);
-      __threadfence();
-      __syncwarp(gmask);
-    } else {
-      // empty sub-block: still keep the column's visit order
-      while (ld_acquire(tickets + col) != tgt) __nanosleep(32);
-    }
-    if (gl == 0) st_release(tickets + col, tgt + 1);
+    ticket_acquire(tickets + col, tgt);     // (empty sub-blocks still keep the visit order)
+    if (n > 0) run_subblock_ring<T, K, L, RS, F>(slots, dup, lo, n, P, Q, g, cp, cq, gl, gmask, ring);
+    ticket_release(tickets + col, tgt + 1, gmask, gl);
   }
 }
 
