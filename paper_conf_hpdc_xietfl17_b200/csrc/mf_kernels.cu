@@ -7,6 +7,8 @@
 
 namespace mfb {
 
+constexpr int kRingSlots = 16, kRingAhead = 7;   // wavefront ring: RS, F -> history window W = 8
+
 // ---------------------------------------------------------------------------------------------
 // batch-Hogwild! (section 5.1).  A worker is a group of L lanes; a warp holds
 // 32/L workers which claim consecutive entries of the epoch's chunk list with ONE atomicAdd per
@@ -144,7 +146,8 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     const int64_t lo = __ldg(sub_off + sb);
     const int n = (int)(__ldg(sub_off + sb + 1) - lo);
     ticket_acquire(tickets + col, tgt);     // (empty sub-blocks still keep the visit order)
-    if (n > 0) run_subblock_ring<T, K, L, RS, F>(slots, dup, lo, n, P, Q, g, cp, cq, gl, gmask, ring);
+    if (n > 0)
+      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo, n, P, Q, g, cp, cq, gl, gbase, gmask, ring);
     ticket_release(tickets + col, tgt + 1, gmask, gl);
   }
 }
@@ -263,7 +266,6 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
 }
 
 
-constexpr int kRingSlots = 16, kRingAhead = 7;   // RS, F  ->  history window W = 8
 
 template <typename T, int K, int L>
 static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
@@ -333,7 +335,9 @@ static cudaError_t rmse_k(const RmseLaunch& a) {
 template <typename T, int K>
 static cudaError_t wavefront_k(const WavefrontLaunch& a) {
   constexpr int S = (int)sizeof(T);
-  if (a.variant == 1 && a.dup) return launch_wavefront2_t<T, K, lanes_for(K, S, 32)>(a);
+  constexpr int L2 = lanes_for(K, S, 32);
+  if constexpr (L2 > kRingAhead && (K * S / L2) % 16 == 0)   // ring kernel needs F < L, 16-B pieces
+    if (a.variant == 1 && a.dup) return launch_wavefront2_t<T, K, L2>(a);
   return launch_wavefront_t<T, K, lanes_for(K, S, 8)>(a);
 }
 
