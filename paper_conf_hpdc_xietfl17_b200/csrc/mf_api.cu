@@ -908,7 +908,8 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
   if (c->wf && c->p.wf_kernel != 2) {
     TRY(c->alloc(&c->dup, (size_t)std::max<int64_t>(c->nslots, 1)));
     if (N > 0) {
-      k_dupdist<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(c->slots, N, Gd, ring_window(), c->dup);
+      k_dupdist<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(c->slots, N, Gd,
+                                                          ring_window(c->k, c->p.storage), c->dup);
       KERNEL_TRY(c);
     }
   }

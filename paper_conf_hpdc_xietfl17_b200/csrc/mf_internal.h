@@ -61,6 +61,6 @@ struct RmseLaunch {
 cudaError_t launch_hogwild(const HogwildLaunch& a);
 cudaError_t launch_wavefront(const WavefrontLaunch& a);
 cudaError_t launch_rmse(const RmseLaunch& a);
-int ring_window();  // W of k_wavefront2
+int ring_window(int k, int storage);  // history window W of k_wavefront2 for this geometry
 
 }  // namespace mfb

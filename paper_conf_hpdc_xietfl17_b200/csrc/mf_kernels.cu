@@ -7,7 +7,14 @@
 
 namespace mfb {
 
-constexpr int kRingSlots = 16, kRingAhead = 7;   // wavefront ring: RS, F -> history window W = 8
+// wavefront ring geometry per (k, storage): rows of K*S bytes, 16 B per lane.  Prefetch F
+// samples ahead in a ring of RS slots (history window W = RS - F - 1); deep (32/15) when a
+// worker's ring fits in 32 KB, else 16/7.  The ring kernel needs F < L (lanes per worker).
+constexpr int ring_lanes(int K, int S) { return (K * S / 16) >= 32 ? 32 : (K * S / 16); }
+constexpr int ring_slots(int K, int S) {
+  return (32 * 2 * K * S <= 32768 && ring_lanes(K, S) > 15) ? 32 : 16;
+}
+constexpr int ring_ahead(int K, int S) { return ring_slots(K, S) == 32 ? 15 : 7; }
 
 // ---------------------------------------------------------------------------------------------
 // batch-Hogwild! (section 5.1).  A worker is a group of L lanes; a warp holds
@@ -269,11 +276,13 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
 
 template <typename T, int K, int L>
 static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
-  auto kern = k_wavefront2<T, K, L, kRingSlots, kRingAhead>;
-  constexpr int ROWB = K * (int)sizeof(T);
+  constexpr int S = (int)sizeof(T);
+  constexpr int RS = ring_slots(K, S), F = ring_ahead(K, S);
+  auto kern = k_wavefront2<T, K, L, RS, F>;
+  constexpr int ROWB = K * S;
   const int threads = 32;                                    // one warp: 32/L workers
   const int wpc = threads / L;
-  const size_t smem = (size_t)wpc * kRingSlots * 2 * ROWB;
+  const size_t smem = (size_t)wpc * RS * 2 * ROWB;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   const int blocks = (int)cdiv64((int64_t)a.s, wpc);
@@ -335,8 +344,8 @@ static cudaError_t rmse_k(const RmseLaunch& a) {
 template <typename T, int K>
 static cudaError_t wavefront_k(const WavefrontLaunch& a) {
   constexpr int S = (int)sizeof(T);
-  constexpr int L2 = lanes_for(K, S, 32);
-  if constexpr (L2 > kRingAhead && (K * S / L2) % 16 == 0)   // ring kernel needs F < L, 16-B pieces
+  constexpr int L2 = ring_lanes(K, S);
+  if constexpr (L2 > ring_ahead(K, S) && (K * S / L2) % 16 == 0)  // needs F < L, 16-B pieces
     if (a.variant == 1 && a.dup) return launch_wavefront2_t<T, K, L2>(a);
   return launch_wavefront_t<T, K, lanes_for(K, S, 8)>(a);
 }
@@ -376,6 +385,15 @@ static cudaError_t wavefront_k(const WavefrontLaunch& a) {
 cudaError_t launch_hogwild(const HogwildLaunch& a) { MF_DISPATCH(hogwild_k, a) }
 cudaError_t launch_wavefront(const WavefrontLaunch& a) { MF_DISPATCH(wavefront_k, a) }
 cudaError_t launch_rmse(const RmseLaunch& a) { MF_DISPATCH(rmse_k, a) }
-int ring_window() { return kRingSlots - kRingAhead - 1; }
+int ring_window(int k, int storage) {
+  const int S = storage == 0 ? 4 : 2;
+  switch (k) {
+    case 16: return ring_slots(16, S) - ring_ahead(16, S) - 1;
+    case 32: return ring_slots(32, S) - ring_ahead(32, S) - 1;
+    case 64: return ring_slots(64, S) - ring_ahead(64, S) - 1;
+    case 128: return ring_slots(128, S) - ring_ahead(128, S) - 1;
+    default: return ring_slots(256, S) - ring_ahead(256, S) - 1;
+  }
+}
 
 }  // namespace mfb
