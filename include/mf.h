@@ -90,8 +90,11 @@ typedef struct mf_params {
                              2 = register pipeline; both give the same result                   */
   int32_t device;         /* CUDA device ordinal                                                */
   int32_t rank, world;    /* world > 1: DSGD strata over `world` GPUs, one ctx per rank         */
-  int32_t transport;      /* 0 = NCCL (world > 1)                                              */
-  const void* nccl_id;    /* 128-byte ncclUniqueId, identical on all ranks (world > 1)          */
+  int32_t transport;      /* world > 1: 0 = NCCL (one process per GPU); 1 = loopback (all ranks
+                             in one process, one host thread each, device-to-device copies;
+                             tests the multi-rank path on one GPU)                              */
+  const void* nccl_id;    /* 128 bytes identical on all ranks (world > 1): the ncclUniqueId, or
+                             for loopback any key naming the group                              */
   void* stream;           /* cudaStream_t or NULL                                               */
   const mf_allocator* alloc; /* NULL = cudaMallocAsync                                          */
 } mf_params;
@@ -174,6 +177,17 @@ mf_status mf_get_stats(mf_ctx* ctx, mf_stats* out);
  * [g*a/G, (g+1)*a/G).  Returns MF_E_INVAL if a % world != 0. */
 mf_status mf_strata_holders(uint64_t seed, int32_t a, int32_t world, int32_t t, int32_t j,
                             int32_t* holder);
+
+/* Host-only plan of sub-epoch j of epoch t for `rank` -- the function mf_train_epoch itself
+ * uses (A: strata order; section 6.1 P:L305-316 adapted).  holders[a] is in/out: on entry the
+ * rank holding each Q segment's valid copy (-1 = every rank holds one), on exit the holders
+ * during sub-epoch j.  Outputs: blocks[*nblocks] (<= a/world) = the strata blocks b = r*a + J
+ * the rank trains; xfers[5 * *nxfers] = {J, src, dst, lo, hi}: segment J (relabelled Q rows
+ * [lo, hi), n = number of columns) moves src -> dst before the sub-epoch.  Caller allocates
+ * blocks[a] and xfers[5a].  MF_E_INVAL for a % world != 0 or n < a. */
+mf_status mf_strata_plan(uint64_t seed, int32_t a, int32_t world, int32_t rank, int64_t n,
+                         int32_t t, int32_t j, int32_t* holders, int64_t* blocks,
+                         int32_t* nblocks, int64_t* xfers, int32_t* nxfers);
 
 void mf_destroy(mf_ctx* ctx);
 const char* mf_last_error(const mf_ctx* ctx);

@@ -111,6 +111,16 @@ __global__ void k_build_test(const int32_t* __restrict__ u, const int32_t* __res
   }
 }
 
+// world > 1: a test rating is evaluated by the rank owning its row segment
+__global__ void k_own_rows(const Rating* __restrict__ t, int64_t N, int64_t m, int64_t a,
+                           int64_t lo_seg, int64_t hi_seg, char* __restrict__ flag) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = (int64_t)t[i].u * a / m;
+    flag[i] = (r >= lo_seg && r < hi_seg) ? 1 : 0;
+  }
+}
+
 __global__ void k_histogram(const uint32_t* __restrict__ bucket, int64_t N,
                             unsigned int* __restrict__ cnt) {
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < N;
@@ -561,6 +571,38 @@ mf_status mf_strata_holders(uint64_t seed, int32_t a, int32_t world, int32_t t, 
   return MF_OK;
 }
 
+mf_status mf_strata_plan(uint64_t seed, int32_t a, int32_t world, int32_t rank, int64_t n,
+                         int32_t t, int32_t j, int32_t* holders, int64_t* blocks,
+                         int32_t* nblocks, int64_t* xfers, int32_t* nxfers) {
+  if (!holders || !blocks || !nblocks || !xfers || !nxfers || rank < 0 || rank >= world || n < a)
+    return MF_E_INVAL;
+  std::vector<int32_t> next((size_t)std::max(a, 1));
+  mf_status s = mf_strata_holders(seed, a, world, t, j, next.data());
+  if (s != MF_OK) return s;
+  const std::vector<int64_t> pi = host_perm(make_stream(seed, kTagStrata, (uint64_t)t, 0), a);
+  // A: rank g owns row segments [g a/G, (g+1) a/G); in sub-epoch j row segment r trains
+  // block (r, (r + pi_t[j]) mod a)
+  const int per = a / world;
+  *nblocks = 0;
+  for (int r = rank * per; r < (rank + 1) * per; ++r)
+    blocks[(*nblocks)++] = (int64_t)r * a + (r + pi[(size_t)j]) % a;
+  // a segment moves iff its valid copy is on one rank (>= 0) that is not the next holder;
+  // segment J = relabelled Q rows [ceil(J n / a), ceil((J+1) n / a))
+  *nxfers = 0;
+  for (int J = 0; J < a; ++J) {
+    if (holders[J] >= 0 && holders[J] != next[(size_t)J]) {
+      int64_t* x = xfers + 5 * (*nxfers)++;
+      x[0] = J;
+      x[1] = holders[J];
+      x[2] = next[(size_t)J];
+      x[3] = cdiv64((int64_t)J * n, a);
+      x[4] = cdiv64((int64_t)(J + 1) * n, a);
+    }
+    holders[J] = next[(size_t)J];
+  }
+  return MF_OK;
+}
+
 mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (!out) return MF_E_INVAL;
   *out = nullptr;
@@ -575,6 +617,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->lane_bytes != 0 && p->lane_bytes != 16 && p->lane_bytes != 32) return MF_E_INVAL;
   if (p->prefetch < 0 || p->prefetch > 2) return MF_E_INVAL;
   if (p->wf_kernel < 0 || p->wf_kernel > 2) return MF_E_INVAL;
+  if (p->transport < 0 || p->transport > 1) return MF_E_INVAL;
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
   const int a = p->grid_a > 0 ? p->grid_a : (world == 1 ? 1 : 8);
@@ -633,7 +676,8 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
     if (!p->nccl_id) { mf_destroy(c); return MF_E_INVAL; }
     std::memcpy(c->nccl_id, p->nccl_id, 128);
     std::string why;
-    c->comm = mf::Comm::create(c->nccl_id, world, p->rank, c->st, &why);
+    c->comm = p->transport == 1 ? mf::Comm::create_loopback(c->nccl_id, world, p->rank, c->st, &why)
+                                : mf::Comm::create(c->nccl_id, world, p->rank, c->st, &why);
     if (!c->comm) {
       c->fail(MF_E_NCCL, "NCCL init failed: %s", why.c_str());
       mf_destroy(c);
@@ -935,6 +979,30 @@ static mf_status load_test(mf_ctx* c, int64_t N, const int32_t* u, const int32_t
     KERNEL_TRY(c);
   }
   c->release(ou); c->release(ov); c->release(orr);
+  if (c->G > 1 && N > 0) {
+    // keep only the test ratings of this rank's row segments (SSE and count are all-reduced)
+    char* flag = nullptr;
+    Rating* kept = nullptr;
+    int64_t* nsel = nullptr;
+    TRY(c->alloc(&flag, (size_t)N));
+    TRY(c->alloc(&kept, (size_t)N));
+    TRY(c->alloc(&nsel, 1));
+    k_own_rows<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(c->test, N, c->m, c->a, c->lo_row_seg(),
+                                                          c->hi_row_seg(), flag);
+    KERNEL_TRY(c);
+    size_t bytes = 0;
+    CUDA_TRY(c, cub::DeviceSelect::Flagged(nullptr, bytes, c->test, flag, kept, nsel, N, c->st));
+    TRY(c->need_tmp(bytes));
+    CUDA_TRY(c, cub::DeviceSelect::Flagged(c->tmp, bytes, c->test, flag, kept, nsel, N, c->st));
+    int64_t h = 0;
+    CUDA_TRY(c, cudaMemcpyAsync(&h, nsel, 8, cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    c->release(c->test);
+    c->release(flag);
+    c->release(nsel);
+    c->test = kept;
+    N = h;
+  }
   CUDA_TRY(c, cudaStreamSynchronize(c->st));
   c->Ntest = N;
   c->test_loaded = true;
@@ -1044,10 +1112,7 @@ static cudaEvent_t ev_at(mf_ctx* c, int i) {
 }
 
 // One strata block set (the blocks rank g trains in sub-epoch j) of epoch t.
-static mf_status run_stratum(mf_ctx* c, int32_t t, int j, const std::vector<int64_t>& pi, float g) {
-  std::vector<int64_t> blocks;
-  for (int r = c->lo_row_seg(); r < c->hi_row_seg(); ++r)
-    blocks.push_back((int64_t)r * c->a + (r + pi[(size_t)j]) % c->a);
+static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, float g) {
   if (!c->wf) {
     ChunkSegs segs{};
     segs.n = 0;
@@ -1114,19 +1179,20 @@ static void q_segment(const mf_ctx* c, int J, char** ptr, size_t* bytes) {
   *bytes = (size_t)(hi - lo) * row_bytes;
 }
 
-// Move every Q segment whose holder changes from `from` to `to` (north_star (5): NCCL
-// send/recv of Q column-segments between sub-epochs).  from[J] < 0: every rank already holds
-// a valid copy, nothing moves.
-static mf_status rotate_q(mf_ctx* c, const int32_t* from, const int32_t* to) {
-  if (c->G == 1) return MF_OK;
+// Move the Q segments of a sub-epoch plan (north_star (5): NCCL send/recv of Q column
+// segments between sub-epochs); xf = {J, src, dst, lo, hi} per transfer (mf_strata_plan).
+static mf_status rotate_q(mf_ctx* c, const int64_t* xf, int nx) {
+  if (c->G == 1 || nx == 0) return MF_OK;
   std::vector<mf::Xfer> xs;
-  for (int J = 0; J < c->a; ++J) {
-    if (from[J] < 0 || from[J] == to[J]) continue;
-    mf::Xfer x;
-    q_segment(c, J, (char**)&x.ptr, &x.bytes);
-    x.src = from[J];
-    x.dst = to[J];
-    xs.push_back(x);
+  const size_t row_bytes = (size_t)c->k * c->ssize();
+  for (int i = 0; i < nx; ++i) {
+    const int64_t* x = xf + 5 * i;
+    mf::Xfer e;
+    e.ptr = (char*)c->Q + (size_t)x[3] * row_bytes;
+    e.bytes = (size_t)(x[4] - x[3]) * row_bytes;
+    e.src = (int)x[1];
+    e.dst = (int)x[2];
+    xs.push_back(e);
   }
   std::string why;
   if (!c->comm->exchange(xs, c->rank, &why)) return c->fail(MF_E_NCCL, "Q rotation: %s", why.c_str());
@@ -1166,19 +1232,27 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   CUDA_TRY(c, cudaEventRecord(c->ev_s0, c->st));
   TRY(build_schedule(c, t));
   CUDA_TRY(c, cudaEventRecord(c->ev_s1, c->st));
-  const std::vector<int64_t> pi = host_perm(make_stream(c->p.seed, kTagStrata, (uint64_t)t, 0), c->a);
-  std::vector<int32_t> hold((size_t)c->a), next((size_t)c->a);
+  // holders of every Q segment's valid copy persist across sub-epochs and epochs (comm);
+  // world == 1 keeps a local vector (every segment is always on rank 0: no transfers)
+  std::vector<int32_t> local_hold((size_t)c->a, -1);
+  int32_t* hold = local_hold.data();
+  std::vector<int32_t> hcopy;
+  if (c->G > 1) {
+    const int32_t* h = c->comm->holders(c->a);
+    hcopy.assign(h, h + c->a);
+    hold = hcopy.data();
+  }
+  std::vector<int64_t> blocks((size_t)c->a), xf((size_t)(5 * c->a));
   CUDA_TRY(c, cudaEventRecord(c->ev_c0, c->st));
   CUDA_TRY(c, cudaEventRecord(c->ev_c1, c->st));
   for (int j = 0; j < c->a; ++j) {
-    if (c->G > 1) {
-      // before sub-epoch j: move every segment whose holder changes (holders of the previous
-      // sub-epoch -- or of the previous epoch's last one -- are tracked in comm)
-      mf_strata_holders(c->p.seed, c->a, c->G, t, j, next.data());
-      TRY(rotate_q(c, c->comm->holders(c->a), next.data()));
-      c->comm->set_holders(next.data(), c->a);
-    }
-    TRY(run_stratum(c, t, j, pi, g));
+    int32_t nb = 0, nx = 0;
+    if (mf_strata_plan(c->p.seed, c->a, c->G, c->rank, c->n, t, j, hold, blocks.data(), &nb,
+                       xf.data(), &nx) != MF_OK)
+      return c->fail(MF_E_INVAL, "strata plan failed");
+    TRY(rotate_q(c, xf.data(), nx));
+    if (c->G > 1) c->comm->set_holders(hold, c->a);
+    TRY(run_stratum(c, std::vector<int64_t>(blocks.begin(), blocks.begin() + nb), g));
   }
   CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
   c->t = t + 1;

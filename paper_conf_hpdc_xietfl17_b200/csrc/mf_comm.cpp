@@ -4,7 +4,10 @@
 #include <dlfcn.h>
 #include <nccl.h>
 
+#include <condition_variable>
 #include <cstring>
+#include <map>
+#include <memory>
 #include <mutex>
 
 namespace mf {
@@ -64,6 +67,77 @@ bool check(Nccl* L, ncclResult_t r, const char* what, std::string* why) {
 
 }  // namespace
 
+// ---------------------------------------------------------------------------------------------
+// loopback transport
+// ---------------------------------------------------------------------------------------------
+struct LoopGroup {
+  int world = 0;
+  std::mutex mu;
+  std::condition_variable cv;
+  int arrived = 0;
+  uint64_t gen = 0;
+  int joined = 0;
+  std::vector<cudaEvent_t> ev;                 // each rank's "my stream reached here" event
+  std::vector<std::vector<void*>> ptrs;        // published device pointers per rank
+
+  void barrier() {
+    std::unique_lock<std::mutex> l(mu);
+    const uint64_t g = gen;
+    if (++arrived == world) {
+      arrived = 0;
+      ++gen;
+      cv.notify_all();
+    } else {
+      cv.wait(l, [&] { return gen != g; });
+    }
+  }
+};
+
+namespace {
+std::mutex g_reg_mu;
+std::map<std::string, std::shared_ptr<LoopGroup>> g_reg;
+
+bool cuda_ok(cudaError_t e, const char* what, std::string* why) {
+  if (e == cudaSuccess) return true;
+  if (why) *why = std::string(what) + ": " + cudaGetErrorString(e);
+  return false;
+}
+}  // namespace
+
+Comm* Comm::create_loopback(const uint8_t id[128], int world, int rank, cudaStream_t st,
+                            std::string* why) {
+  const std::string key(reinterpret_cast<const char*>(id), 128);
+  std::shared_ptr<LoopGroup> g;
+  {
+    std::lock_guard<std::mutex> l(g_reg_mu);
+    auto& slot = g_reg[key];
+    if (!slot) {
+      slot = std::make_shared<LoopGroup>();
+      slot->world = world;
+      slot->ev.assign((size_t)world, nullptr);
+      slot->ptrs.assign((size_t)world, {});
+    }
+    g = slot;
+    if (g->world != world) {
+      if (why) *why = "loopback group world size mismatch";
+      return nullptr;
+    }
+    ++g->joined;
+  }
+  Comm* c = new Comm();
+  c->loop_ = g.get();
+  c->st_ = st;
+  c->world_ = world;
+  c->rank_ = rank;
+  if (!cuda_ok(cudaEventCreateWithFlags(&c->ev_, cudaEventDisableTiming), "cudaEventCreate", why)) {
+    delete c;
+    return nullptr;
+  }
+  g->ev[(size_t)rank] = c->ev_;
+  g->barrier();                                // all ranks joined (like ncclCommInitRank)
+  return c;
+}
+
 Comm* Comm::create(const uint8_t id[128], int world, int rank, cudaStream_t st, std::string* why) {
   Nccl* L = nccl(why);
   if (!L) return nullptr;
@@ -82,6 +156,17 @@ Comm* Comm::create(const uint8_t id[128], int world, int rank, cudaStream_t st, 
 
 void Comm::destroy(Comm* c) {
   if (!c) return;
+  if (c->loop_) {
+    std::lock_guard<std::mutex> l(g_reg_mu);
+    for (auto it = g_reg.begin(); it != g_reg.end(); ++it)
+      if (it->second.get() == c->loop_ && --it->second->joined == 0) {
+        g_reg.erase(it);
+        break;
+      }
+    if (c->ev_) cudaEventDestroy(c->ev_);
+    delete c;
+    return;
+  }
   Nccl* L = nccl(nullptr);
   if (L && c->comm_) L->CommDestroy(static_cast<ncclComm_t>(c->comm_));
   delete c;
@@ -89,6 +174,29 @@ void Comm::destroy(Comm* c) {
 
 bool Comm::exchange(const std::vector<Xfer>& xs, int me, std::string* why) {
   if (xs.empty()) return true;
+  if (loop_) {
+    LoopGroup& g = *loop_;
+    std::vector<void*> mine;
+    for (const Xfer& x : xs) mine.push_back(x.ptr);
+    g.ptrs[(size_t)me] = mine;
+    if (!cuda_ok(cudaEventRecord(ev_, st_), "cudaEventRecord", why)) return false;
+    g.barrier();                               // every rank's segments are final on its stream
+    for (size_t i = 0; i < xs.size(); ++i)
+      if (xs[i].dst == me) {
+        if (!cuda_ok(cudaStreamWaitEvent(st_, g.ev[(size_t)xs[i].src], 0), "wait", why)) return false;
+        if (!cuda_ok(cudaMemcpyAsync(xs[i].ptr, g.ptrs[(size_t)xs[i].src][i], xs[i].bytes,
+                                     cudaMemcpyDeviceToDevice, st_), "copy", why))
+          return false;
+      }
+    g.barrier();                               // all copies enqueued before events are re-recorded
+    if (!cuda_ok(cudaEventRecord(ev_, st_), "cudaEventRecord", why)) return false;
+    g.barrier();
+    for (size_t i = 0; i < xs.size(); ++i)     // a source does not overwrite before the copy ran
+      if (xs[i].src == me && !cuda_ok(cudaStreamWaitEvent(st_, g.ev[(size_t)xs[i].dst], 0), "wait", why))
+        return false;
+    g.barrier();
+    return true;
+  }
   Nccl* L = nccl(why);
   if (!L) return false;
   ncclComm_t cm = static_cast<ncclComm_t>(comm_);
@@ -103,6 +211,12 @@ bool Comm::exchange(const std::vector<Xfer>& xs, int me, std::string* why) {
 }
 
 bool Comm::broadcast(void* ptr, size_t bytes, int root, std::string* why) {
+  if (loop_) {
+    std::vector<Xfer> xs;
+    for (int r = 0; r < world_; ++r)
+      if (r != root) xs.push_back(Xfer{ptr, bytes, root, r});
+    return exchange(xs, rank_, why);
+  }
   Nccl* L = nccl(why);
   if (!L) return false;
   return check(L, L->Bcast(ptr, ptr, bytes, ncclUint8, root, static_cast<ncclComm_t>(comm_), st_),
@@ -110,6 +224,28 @@ bool Comm::broadcast(void* ptr, size_t bytes, int root, std::string* why) {
 }
 
 bool Comm::allreduce_sum(double* dptr, size_t n, std::string* why) {
+  if (loop_) {
+    LoopGroup& g = *loop_;
+    g.ptrs[(size_t)rank_] = {dptr};
+    if (!cuda_ok(cudaEventRecord(ev_, st_), "cudaEventRecord", why)) return false;
+    g.barrier();
+    std::vector<double> acc(n, 0.0), tmp(n);
+    for (int r = 0; r < world_; ++r) {         // fixed rank order: identical sum on every rank
+      if (!cuda_ok(cudaStreamWaitEvent(st_, g.ev[(size_t)r], 0), "wait", why)) return false;
+      if (!cuda_ok(cudaMemcpyAsync(tmp.data(), g.ptrs[(size_t)r][0], n * sizeof(double),
+                                   cudaMemcpyDeviceToHost, st_), "copy", why) ||
+          !cuda_ok(cudaStreamSynchronize(st_), "sync", why))
+        return false;
+      for (size_t i = 0; i < n; ++i) acc[i] += tmp[i];
+    }
+    g.barrier();                               // everyone read every input before overwriting
+    if (!cuda_ok(cudaMemcpyAsync(dptr, acc.data(), n * sizeof(double), cudaMemcpyHostToDevice, st_),
+                 "copy", why) ||
+        !cuda_ok(cudaStreamSynchronize(st_), "sync", why))
+      return false;
+    g.barrier();
+    return true;
+  }
   Nccl* L = nccl(why);
   if (!L) return false;
   return check(L, L->AllReduce(dptr, dptr, n, ncclFloat64, ncclSum, static_cast<ncclComm_t>(comm_), st_),

@@ -19,9 +19,19 @@ struct Xfer {
   int src, dst;
 };
 
+struct LoopGroup;
+
+// Two transports behind one interface:
+//  * NCCL (transport 0): one process per GPU, libnccl.so.2 dlopen'ed.
+//  * loopback (transport 1, tests): all ranks are ctxs of ONE process driven by one host thread
+//    each (any devices, e.g. all on one GPU); transfers are stream-ordered device-to-device
+//    copies, synchronised with CUDA events and a host barrier.  Same protocol and plan, so the
+//    multi-rank path is testable on a single GPU.
 class Comm {
  public:
   static Comm* create(const uint8_t id[128], int world, int rank, cudaStream_t st, std::string* why);
+  static Comm* create_loopback(const uint8_t id[128], int world, int rank, cudaStream_t st,
+                               std::string* why);
   static void destroy(Comm* c);
 
   // One grouped set of point-to-point transfers (ncclGroupStart/ncclSend/ncclRecv/ncclGroupEnd).
@@ -43,6 +53,8 @@ class Comm {
  private:
   Comm() = default;
   void* comm_ = nullptr;
+  LoopGroup* loop_ = nullptr;
+  cudaEvent_t ev_ = nullptr;
   cudaStream_t st_ = nullptr;
   int world_ = 1, rank_ = 0;
   std::vector<int32_t> holders_;

@@ -67,7 +67,8 @@ class Stats(ctypes.Structure):
 _lib = None
 EXPORTED = ["mf_abi_version", "mf_params_default", "mf_create", "mf_load_coo", "mf_train_epoch",
             "mf_rmse", "mf_get_factors", "mf_set_factors", "mf_set_epoch", "mf_get_epoch",
-            "mf_export_schedule", "mf_get_stats", "mf_strata_holders", "mf_destroy",
+            "mf_export_schedule", "mf_get_stats", "mf_strata_holders", "mf_strata_plan",
+            "mf_destroy",
             "mf_last_error", "mf_status_string"]
 
 
@@ -95,6 +96,7 @@ def lib() -> ctypes.CDLL:
         "mf_export_schedule": (i32, [vp, i32, i32, vp, ctypes.POINTER(i64)]),
         "mf_get_stats": (i32, [vp, ctypes.POINTER(Stats)]),
         "mf_strata_holders": (i32, [u64, i32, i32, i32, i32, vp]),
+        "mf_strata_plan": (i32, [u64, i32, i32, i32, i64, i32, i32, vp, vp, vp, vp, vp]),
         "mf_destroy": (None, [vp]),
         "mf_last_error": (ctypes.c_char_p, [vp]),
         "mf_status_string": (ctypes.c_char_p, [i32]),
@@ -114,6 +116,21 @@ def strata_holders(seed: int, a: int, world: int, t: int, j: int) -> list[int]:
     if st != 0:
         raise MFError(st, "mf_strata_holders")
     return list(out)
+
+
+def strata_plan(seed: int, a: int, world: int, rank: int, n: int, t: int, j: int, holders):
+    """Host-only plan of sub-epoch j (the one mf_train_epoch executes): returns
+    (blocks, transfers, new_holders); transfers = [(J, src, dst, lo, hi), ...]."""
+    h = (ctypes.c_int32 * a)(*holders)
+    blocks = (ctypes.c_int64 * a)()
+    xf = (ctypes.c_int64 * (5 * a))()
+    nb, nx = ctypes.c_int32(0), ctypes.c_int32(0)
+    st = lib().mf_strata_plan(seed, a, world, rank, n, t, j, h, blocks, ctypes.byref(nb), xf,
+                              ctypes.byref(nx))
+    if st != 0:
+        raise MFError(st, "mf_strata_plan")
+    tr = [tuple(xf[5 * i:5 * i + 5]) for i in range(nx.value)]
+    return list(blocks[:nb.value]), tr, list(h)
 
 
 def _torch():
@@ -166,7 +183,8 @@ class MF:
                  schedule: str = "hogwild", storage: str = "fp32", workers: int = 0,
                  batch_f: int = 256, wf_cols: int = 0, grid_a: int = 0, cyclic: bool = False,
                  lane_bytes: int = 0, prefetch: int = 0, wf_kernel: int = 0, device: int = 0, rank: int = 0, world: int = 1,
-                 nccl_id: bytes | None = None, stream=None, allocator: str = "torch"):
+                 nccl_id: bytes | None = None, transport: int = 0, stream=None,
+                 allocator: str = "torch"):
         L = lib()
         p = Params()
         L.mf_params_default(ctypes.byref(p))
@@ -178,7 +196,7 @@ class MF:
         p.schedule, p.storage = SCHEDULE[schedule], STORAGE[storage]
         p.workers, p.batch_f, p.wf_cols, p.grid_a = workers, batch_f, wf_cols, grid_a
         p.cyclic, p.lane_bytes, p.prefetch, p.wf_kernel = int(cyclic), lane_bytes, prefetch, wf_kernel
-        p.device, p.rank, p.world = device, rank, world
+        p.device, p.rank, p.world, p.transport = device, rank, world, transport
         self._id_buf = None
         if nccl_id is not None:
             self._id_buf = ctypes.create_string_buffer(bytes(nccl_id), 128)
