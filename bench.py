@@ -32,8 +32,8 @@ CPU_SAMPLE = 1 << 23        # oracle sample (ratings) for cpu_baseline
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
-    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="mf", choices=["mf", "reference"])
     ap.add_argument("--workload", default="netflix", choices=["netflix", "yahoo", "hugewiki", "tiny"])
     ap.add_argument("--storage", default="fp16", choices=["fp16", "fp32", "bf16"])
@@ -182,7 +182,7 @@ def run_reference(args):
         return
     device = "cuda" if torch.cuda.is_available() else "cpu"
     R, hp = workload(args, device)
-    per_step = max(1 << 20, args.cpu_sample // 4)
+    per_step = min(1 << 20, args.cpu_sample)
     vals = []
     for i in range(args.warmup + args.steps):
         cb = cpu_baseline(R, hp, args, per_step)
