@@ -638,7 +638,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   c->wf = p->schedule == MF_WAVEFRONT;
   if (c->wf) {
     const int64_t rows_per_seg = p->m / a;
-    int64_t s = p->workers > 0 ? p->workers : std::min<int64_t>(1024, std::max<int64_t>(1, rows_per_seg / 4));
+    int64_t s = p->workers > 0 ? p->workers : std::min<int64_t>(768, std::max<int64_t>(1, rows_per_seg / 4));
     c->s = (int)s;
     c->c = p->wf_cols > 0 ? p->wf_cols : 2 * c->s;
     if (p->cyclic && c->c < c->s) { delete c; return MF_E_INVAL; }

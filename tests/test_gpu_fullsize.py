@@ -86,7 +86,7 @@ def test_fullsize_hogwild_full_concurrency_converges_like_serial(netflix):
     res = {}
     for sched in ("hogwild", "wavefront"):
         g = mf.MF(R.m, R.n, 128, storage="fp32", schedule=sched, seed=SEED,
-                  workers=2048 if sched == "wavefront" else 0, **HP)
+                  workers=768 if sched == "wavefront" else 0, **HP)
         g.load(R.u, R.v, R.r)
         g.load(R.ut, R.vt, R.rt, "test")
         for _ in range(20):
@@ -101,7 +101,7 @@ def test_fullsize_wavefront_deterministic_rerun(netflix):
     R = netflix
     outs = []
     for _ in range(2):
-        g = mf.MF(R.m, R.n, 128, storage="fp32", schedule="wavefront", workers=2048, seed=SEED, **HP)
+        g = mf.MF(R.m, R.n, 128, storage="fp32", schedule="wavefront", workers=768, seed=SEED, **HP)
         g.load(R.u, R.v, R.r)
         g.train_epoch()
         outs.append(g.factors())
