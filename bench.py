@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-deterministic", action="store_true",
+                    help="skip the extra deterministic-wavefront line (north_star target run)")
     ap.add_argument("--cpu-sample", type=int, default=CPU_SAMPLE)
     return ap.parse_args()
 
@@ -281,6 +283,9 @@ def main():
     e2e = None
     if not args.no_e2e and world == 1:
         e2e = run_e2e(args, R, kw, stream)
+    det = None
+    if not args.no_deterministic and world == 1 and args.schedule == "hogwild":
+        det = run_deterministic(args, R, hp, stream)
     cpu = None
     if not args.no_cpu_baseline and world == 1 and rank == 0:
         cpu = cpu_baseline(R, hp, args, args.cpu_sample)
@@ -294,13 +299,51 @@ def main():
                 "sec_per_epoch": ms_step / 1000.0, "test_rmse": rmse, "test_rmse_init": rmse0,
                 "epochs_trained": args.warmup + args.steps,
                 "gpu_launches": int(launches), "roofline": roof, "clocks": clk.summary(),
-                "e2e": e2e, "cpu_baseline": cpu,
+                "e2e": e2e, "cpu_baseline": cpu, "deterministic": det,
                 "paper_context": "cuMF_SGD Table 5 (P:L414-415), Netflix fp16 Hogwild: 267M/s "
                                  "TITAN X, 613M/s P100 (other hardware; context only)"}
         print(json.dumps(line), flush=True)
     if world > 1:
         import torch.distributed as dist
         dist.destroy_process_group()
+
+
+def run_deterministic(args, R, hp, stream):
+    """The north_star target run: the deterministic conflict-free wavefront (oracle-exact
+    order), fp32 storage, k = args.k, s = 768 workers, cyclic column order with c = 8s
+    (SURVEY App. A cyclic variant), on the same data; device-timed like the main line."""
+    from paper_conf_hpdc_xietfl17_b200 import mf
+    steps, warm = max(3, args.steps // 2), 2
+    m = mf.MF(R.m, R.n, args.k, stream=stream, schedule="wavefront", storage="fp32", workers=768,
+              wf_cols=6144, cyclic=True, seed=42, **hp)
+    m.load(R.u, R.v, R.r, "train")
+    m.load(R.ut, R.vt, R.rt, "test")
+    for _ in range(warm):
+        m.train_epoch()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    sgd, upd = [], 0
+    e0.record(stream)
+    for _ in range(steps):
+        m.train_epoch()
+        st = m.stats()
+        sgd.append(st["sgd_ms"])
+        upd += st["updates"]
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    hbm, _ = peaks()
+    bpu = st["bytes_per_update"]
+    achieved = upd * bpu / (float(np.sum(sgd)) / 1000.0) / 1e9
+    out = {"schedule": "wavefront (deterministic, cyclic, s=768, c=6144)", "storage": "fp32",
+           "value": upd / (ms / 1000.0), "unit": "updates/s", "ms_per_step": ms / steps,
+           "steps": steps, "warmup": warm, "test_rmse": m.rmse("test"),
+           "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                        "frac": achieved / hbm, "bytes_per_update": bpu,
+                        "step_frac": upd / (ms / 1000.0) * bpu / 1e9 / hbm}}
+    m.close()
+    return out
 
 
 def run_e2e(args, R, kw, stream):

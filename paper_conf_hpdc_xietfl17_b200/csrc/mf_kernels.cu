@@ -139,8 +139,11 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
   const int lane = threadIdx.x & 31;
   const int grp = lane / L, gl = lane % L, gbase = grp * L;
   const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
-  const int local = threadIdx.x / L;
-  const int worker = blockIdx.x * (blockDim.x / L) + local;
+  // one worker per warp (lanes >= L idle): two workers sharing a warp would diverge (each
+  // spins on its own ticket) and serialise each other's instruction streams
+  if (lane >= L) return;
+  const int local = threadIdx.x >> 5;
+  const int worker = blockIdx.x * (blockDim.x >> 5) + local;
   if (worker >= s) return;
   char* ring = smem + (size_t)local * RS * 2 * ROWB;
   const float cp = 1.f - g * lp, cq = 1.f - g * lq;
@@ -280,8 +283,8 @@ static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
   constexpr int RS = ring_slots(K, S), F = ring_ahead(K, S);
   auto kern = k_wavefront2<T, K, L, RS, F>;
   constexpr int ROWB = K * S;
-  const int threads = 32;                                    // one warp: 32/L workers
-  const int wpc = threads / L;
+  const int threads = 32;                                    // one warp = one worker
+  const int wpc = 1;
   const size_t smem = (size_t)wpc * RS * 2 * ROWB;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
