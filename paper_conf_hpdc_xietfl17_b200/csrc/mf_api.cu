@@ -1149,6 +1149,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     WavefrontLaunch L{};
     L.storage = c->p.storage; L.k = c->k; L.slots = c->slots; L.sub_off = c->sub_off + base;
     L.variant = c->p.wf_kernel == 2 ? 0 : 1;
+    L.lane_bytes = c->p.lane_bytes;
     L.dup = c->dup;
     L.seq = c->seq + base; L.rank = c->rank_arr + base; L.tickets = c->tickets;
     L.s = c->s; L.c = c->c; L.num_sms = c->num_sms; L.P = c->P; L.Q = c->Q; L.g = g;

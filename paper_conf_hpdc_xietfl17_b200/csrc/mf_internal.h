@@ -33,6 +33,7 @@ struct HogwildLaunch {
 
 struct WavefrontLaunch {
   int storage, k, variant;  // variant 1 = ring-staged k_wavefront2 (needs dup), 0 = k_wavefront
+  int lane_bytes;           // ring kernel: 16 (default) or 32 bytes per lane
   const Rating* slots;
   const uint16_t* dup;     // per slot: distance to previous same-u (low byte) / same-v (high
                            // byte) sample of the sub-block if <= ring_window(), else 0

@@ -348,6 +348,9 @@ template <typename T, int K>
 static cudaError_t wavefront_k(const WavefrontLaunch& a) {
   constexpr int S = (int)sizeof(T);
   constexpr int L2 = ring_lanes(K, S);
+  constexpr int L3 = L2 / 2;                 // lane_bytes = 32: half the lanes, 32 B per lane
+  if constexpr (L3 > ring_ahead(K, S) && (K * S / L3) % 16 == 0)
+    if (a.variant == 1 && a.dup && a.lane_bytes == 32) return launch_wavefront2_t<T, K, L3>(a);
   if constexpr (L2 > ring_ahead(K, S) && (K * S / L2) % 16 == 0)  // needs F < L, 16-B pieces
     if (a.variant == 1 && a.dup) return launch_wavefront2_t<T, K, L2>(a);
   return launch_wavefront_t<T, K, lanes_for(K, S, 8)>(a);
