@@ -45,6 +45,9 @@ def parse():
     ap.add_argument("--lane-bytes", type=int, default=0)
     ap.add_argument("--prefetch", type=int, default=0)
     ap.add_argument("--wf-kernel", type=int, default=0)
+    ap.add_argument("--staged", action="store_true",
+                    help="out-of-core: ratings in pinned host memory, streamed per stratum")
+    ap.add_argument("--grid-a", type=int, default=0)
     ap.add_argument("--fraction", type=float, default=1.0, help="scale the workload (testing)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -210,6 +213,7 @@ def config_of(args, R):
             "m": R.m, "n": R.n, "N_train": R.N, "N_test": R.Ntest, "k": args.k,
             "storage": args.storage, "schedule": args.schedule, "batch_f": 256,
             "parallelism": f"dsgd-strata{args.gpus}" if args.gpus > 1 else "1gpu",
+            "staged": bool(args.staged), "grid_a": args.grid_a or (8 if args.gpus > 1 else 1),
             "l2": "inputs larger than L2 (COO %.2f GB per epoch); model P+Q stays cached as in "
                   "any training run" % (R.N * 12 / 1e9)}
 
@@ -231,7 +235,7 @@ def main():
         nccl_id = mf.nccl_unique_id_via()
     kw = dict(schedule=args.schedule, storage=args.storage, workers=args.workers,
               wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes, prefetch=args.prefetch,
-              wf_kernel=args.wf_kernel, seed=42,
+              wf_kernel=args.wf_kernel, staged=args.staged, grid_a=args.grid_a, seed=42,
               device=local, rank=rank, world=world, nccl_id=nccl_id, **hp)
     torch.cuda.synchronize()
     model = mf.MF(R.m, R.n, args.k, stream=stream, **kw)

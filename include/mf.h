@@ -86,6 +86,11 @@ typedef struct mf_params {
   int32_t cyclic;         /* wavefront: 1 = cyclic column order (A: cyclic variant), needs c >= s */
   int32_t lane_bytes;     /* Hogwild/RMSE kernel: bytes of p_u (and q_v) per lane, 16 or 32 (0 = 16) */
   int32_t prefetch;       /* Hogwild software-pipeline depth: samples in flight per worker, 1 or 2 (0 = 1) */
+  int32_t staged;         /* 1 = out-of-core ratings (section 6.2): after the GPU
+                             preprocessing the bucketed ratings live in pinned host memory and
+                             each stratum's blocks stream into one of two HBM buffers on a copy
+                             stream while the previous stratum computes; P, Q stay resident.
+                             Same order and result as resident.  0 = ratings resident in HBM */
   int32_t wf_kernel;      /* wavefront kernel: 0 = auto = 1 = ring-staged (cp.async smem ring),
                              2 = register pipeline; both give the same result                   */
   int32_t device;         /* CUDA device ordinal                                                */

@@ -421,6 +421,22 @@ struct mf_ctx {
 
   mf::Comm* comm = nullptr;
 
+  // out-of-core staging (params.staged; section 6.2): the bucketed ratings live in
+  // pinned host memory; each stratum's blocks are copied into one of two device buffers on a
+  // copy stream while the previous stratum computes.
+  bool staged = false;
+  Rating* h_slots = nullptr;
+  uint16_t* h_dup = nullptr;
+  Rating* stg[2] = {nullptr, nullptr};
+  uint16_t* stg_dup[2] = {nullptr, nullptr};
+  int64_t stg_cap = 0;
+  cudaStream_t cs = nullptr;
+  cudaEvent_t ev_h2d[2] = {nullptr, nullptr}, ev_free[2] = {nullptr, nullptr};
+  std::vector<std::pair<int64_t, int64_t>> stg_shift[2];   // (block, slot shift) per buffer
+  int64_t staged_t = -1, staged_j = -1;
+  int cur_buf = 0;
+  int64_t h2d_bytes = 0;
+
   mf_status fail(mf_status s, const char* fmt, ...) {
     char buf[512];
     va_list ap;
@@ -618,6 +634,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->prefetch < 0 || p->prefetch > 2) return MF_E_INVAL;
   if (p->wf_kernel < 0 || p->wf_kernel > 2) return MF_E_INVAL;
   if (p->transport < 0 || p->transport > 1) return MF_E_INVAL;
+  if (p->staged < 0 || p->staged > 1) return MF_E_INVAL;
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
   const int a = p->grid_a > 0 ? p->grid_a : (world == 1 ? 1 : 8);
@@ -636,6 +653,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   c->rank = p->rank;
   c->f = p->batch_f > 0 ? p->batch_f : 256;
   c->wf = p->schedule == MF_WAVEFRONT;
+  c->staged = p->staged == 1;
   if (c->wf) {
     const int64_t rows_per_seg = p->m / a;
     int64_t s = p->workers > 0 ? p->workers : std::min<int64_t>(768, std::max<int64_t>(1, rows_per_seg / 4));
@@ -707,6 +725,14 @@ void mf_destroy(mf_ctx* c) {
   for (cudaEvent_t e : {c->ev_e0, c->ev_e1, c->ev_s0, c->ev_s1, c->ev_c0, c->ev_c1})
     if (e) cudaEventDestroy(e);
   if (c->comm) mf::Comm::destroy(c->comm);
+  if (c->cs) cudaStreamSynchronize(c->cs);
+  if (c->h_slots) cudaFreeHost(c->h_slots);
+  if (c->h_dup) cudaFreeHost(c->h_dup);
+  for (int i = 0; i < 2; ++i) {
+    if (c->ev_h2d[i]) cudaEventDestroy(c->ev_h2d[i]);
+    if (c->ev_free[i]) cudaEventDestroy(c->ev_free[i]);
+  }
+  if (c->cs) cudaStreamDestroy(c->cs);
   if (c->own_stream && c->st) cudaStreamDestroy(c->st);
   cudaGetLastError();
   delete c;
@@ -816,6 +842,79 @@ static mf_status alloc_schedule(mf_ctx* c) {
   } else {
     TRY(c->alloc(&c->chunk_order, (size_t)cap));
   }
+  return MF_OK;
+}
+
+// Move the bucketed ratings (and the wavefront dup metadata) to pinned host memory and size
+// the two device staging buffers for the largest stratum this rank can meet:
+// sum over owned row segments r of max_J |block (r, J)|.
+static mf_status setup_staging(mf_ctx* c) {
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  const size_t ns = (size_t)std::max<int64_t>(c->nslots, 1);
+  CUDA_TRY(c, cudaMallocHost(&c->h_slots, ns * sizeof(Rating)));
+  CUDA_TRY(c, cudaMemcpyAsync(c->h_slots, c->slots, ns * sizeof(Rating), cudaMemcpyDeviceToHost, c->st));
+  if (c->dup) {
+    CUDA_TRY(c, cudaMallocHost(&c->h_dup, ns * sizeof(uint16_t)));
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_dup, c->dup, ns * sizeof(uint16_t), cudaMemcpyDeviceToHost, c->st));
+  }
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  c->release(c->slots);
+  c->release(c->dup);
+  c->release(c->slot_pos);
+  c->release(c->perm);
+  int64_t cap = 1;
+  int64_t sum = 0;
+  for (int r = c->lo_row_seg(); r < c->hi_row_seg(); ++r) {
+    int64_t mx = 0;
+    for (int J = 0; J < c->a; ++J) {
+      const int64_t b = (int64_t)r * c->a + J;
+      mx = std::max(mx, c->blk_off[(size_t)b + 1] - c->blk_off[(size_t)b]);
+    }
+    sum += mx;
+  }
+  cap = std::max<int64_t>(cap, sum);
+  c->stg_cap = cap;
+  for (int i = 0; i < 2; ++i) {
+    TRY(c->alloc(&c->stg[i], (size_t)cap));
+    if (c->h_dup) TRY(c->alloc(&c->stg_dup[i], (size_t)cap));
+    CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_h2d[i], cudaEventDisableTiming));
+    CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_free[i], cudaEventDisableTiming));
+    CUDA_TRY(c, cudaEventRecord(c->ev_free[i], c->st));
+  }
+  CUDA_TRY(c, cudaStreamCreateWithFlags(&c->cs, cudaStreamNonBlocking));
+  return MF_OK;
+}
+
+// The blocks this rank trains in sub-epoch j of epoch t (A: strata order).
+static std::vector<int64_t> stratum_blocks(const mf_ctx* c, int32_t t, int32_t j) {
+  const std::vector<int64_t> pi = host_perm(make_stream(c->p.seed, kTagStrata, (uint64_t)t, 0), c->a);
+  std::vector<int64_t> out;
+  for (int r = c->lo_row_seg(); r < c->hi_row_seg(); ++r)
+    out.push_back((int64_t)r * c->a + (r + pi[(size_t)j]) % c->a);
+  return out;
+}
+
+// Copy the blocks of (t, j) from pinned host memory into staging buffer `buf`, packed, on the
+// copy stream, after the compute stream released the buffer.
+static mf_status stage(mf_ctx* c, int32_t t, int32_t j, int buf) {
+  CUDA_TRY(c, cudaStreamWaitEvent(c->cs, c->ev_free[buf], 0));
+  c->stg_shift[buf].clear();
+  int64_t off = 0;
+  for (int64_t b : stratum_blocks(c, t, j)) {
+    const int64_t lo = c->blk_off[(size_t)b], len = c->blk_off[(size_t)b + 1] - lo;
+    c->stg_shift[buf].push_back({b, off - lo});
+    if (len == 0) continue;
+    CUDA_TRY(c, cudaMemcpyAsync(c->stg[buf] + off, c->h_slots + lo, (size_t)len * sizeof(Rating),
+                                cudaMemcpyHostToDevice, c->cs));
+    if (c->h_dup)
+      CUDA_TRY(c, cudaMemcpyAsync(c->stg_dup[buf] + off, c->h_dup + lo, (size_t)len * 2,
+                                  cudaMemcpyHostToDevice, c->cs));
+    c->h2d_bytes += len * (int64_t)(sizeof(Rating) + (c->h_dup ? 2 : 0));
+    off += len;
+  }
+  CUDA_TRY(c, cudaEventRecord(c->ev_h2d[buf], c->cs));
+  c->staged_t = t;
+  c->staged_j = j;
   return MF_OK;
 }
 
@@ -959,6 +1058,7 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
   }
   TRY(init_factors(c));
   TRY(alloc_schedule(c));
+  if (c->staged) TRY(setup_staging(c));
   CUDA_TRY(c, cudaStreamSynchronize(c->st));
   c->train_loaded = true;
   return MF_OK;
@@ -1112,7 +1212,17 @@ static cudaEvent_t ev_at(mf_ctx* c, int i) {
 }
 
 // One strata block set (the blocks rank g trains in sub-epoch j) of epoch t.
-static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, float g) {
+// shift of block b in the current staging buffer (0 when the ratings are resident)
+static int64_t slot_shift(const mf_ctx* c, int buf, int64_t b) {
+  if (!c->staged) return 0;
+  for (const auto& x : c->stg_shift[buf])
+    if (x.first == b) return x.second;
+  return 0;
+}
+
+static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, float g, int buf) {
+  const Rating* slots = c->staged ? c->stg[buf] : c->slots;
+  const uint16_t* dup = c->staged ? c->stg_dup[buf] : c->dup;
   if (!c->wf) {
     ChunkSegs segs{};
     segs.n = 0;
@@ -1122,6 +1232,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
       if (nch == 0) continue;
       segs.begin[segs.n] = c->ch_off[(size_t)b];
       segs.prefix[segs.n + 1] = segs.prefix[segs.n] + nch;
+      segs.shift[segs.n] = slot_shift(c, buf, b);
       c->updates += c->blk_len[(size_t)b];
       ++segs.n;
     }
@@ -1130,7 +1241,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     HogwildLaunch L{};
     L.storage = c->p.storage; L.k = c->k; L.lane_bytes = c->p.lane_bytes ? c->p.lane_bytes : 16;
     L.prefetch = c->p.prefetch ? c->p.prefetch : 1;
-    L.slots = c->slots; L.chunks = c->chunk_order; L.segs = segs; L.counter = c->counter;
+    L.slots = slots; L.chunks = c->chunk_order; L.segs = segs; L.counter = c->counter;
     L.workers = c->p.workers; L.num_sms = c->num_sms; L.f = c->f;
     L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
     L.out_workers = &c->last_workers; L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
@@ -1147,10 +1258,11 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     CUDA_TRY(c, cudaMemsetAsync(c->tickets, 0, (size_t)c->c * 4, c->st));
     const int64_t base = b * (int64_t)c->s * c->c;
     WavefrontLaunch L{};
-    L.storage = c->p.storage; L.k = c->k; L.slots = c->slots; L.sub_off = c->sub_off + base;
+    L.storage = c->p.storage; L.k = c->k; L.slots = slots; L.sub_off = c->sub_off + base;
+    L.shift = slot_shift(c, buf, b);
     L.variant = c->p.wf_kernel == 2 ? 0 : 1;
     L.lane_bytes = c->p.lane_bytes;
-    L.dup = c->dup;
+    L.dup = dup;
     L.seq = c->seq + base; L.rank = c->rank_arr + base; L.tickets = c->tickets;
     L.s = c->s; L.c = c->c; L.num_sms = c->num_sms; L.P = c->P; L.Q = c->Q; L.g = g;
     L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
@@ -1253,7 +1365,20 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
       return c->fail(MF_E_INVAL, "strata plan failed");
     TRY(rotate_q(c, xf.data(), nx));
     if (c->G > 1) c->comm->set_holders(hold, c->a);
-    TRY(run_stratum(c, std::vector<int64_t>(blocks.begin(), blocks.begin() + nb), g));
+    int buf = 0;
+    if (c->staged) {
+      // stratum (t, j) is normally pre-staged by the previous step (also across epochs)
+      if (c->staged_t != t || c->staged_j != j) TRY(stage(c, t, j, c->cur_buf));
+      buf = c->cur_buf;
+      const bool last = j + 1 == c->a;
+      TRY(stage(c, last ? t + 1 : t, last ? 0 : j + 1, 1 - buf));   // overlap the next copy
+      CUDA_TRY(c, cudaStreamWaitEvent(c->st, c->ev_h2d[buf], 0));
+    }
+    TRY(run_stratum(c, std::vector<int64_t>(blocks.begin(), blocks.begin() + nb), g, buf));
+    if (c->staged) {
+      CUDA_TRY(c, cudaEventRecord(c->ev_free[buf], c->st));
+      c->cur_buf = 1 - buf;
+    }
   }
   CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
   c->t = t + 1;
@@ -1310,8 +1435,8 @@ mf_status mf_rmse(mf_ctx* c, int32_t set, double* out) {
   } else {
     return c->fail(MF_E_INVAL, "bad set");
   }
-  if (set == MF_TRAIN && c->G > 1)
-    return c->fail(MF_E_UNSUPPORTED, "train-set RMSE is single-GPU only");
+  if (set == MF_TRAIN && (c->G > 1 || c->staged))
+    return c->fail(MF_E_UNSUPPORTED, "train-set RMSE needs resident single-GPU ratings");
   // world > 1: every rank evaluates the test samples of the row segments it owns (filtered at
   // load) against a complete Q, then the SSE and count are summed over ranks.
   if (c->G > 1) TRY(gather_q(c));
@@ -1441,6 +1566,8 @@ mf_status mf_export_schedule(mf_ctx* c, int32_t what, int32_t epoch, int64_t* bu
   if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
   const int64_t nb = (int64_t)c->a * c->a;
   int64_t need = 0;
+  if (c->staged && (what == MF_EX_PERM || what == MF_EX_BLOCKID))
+    return c->fail(MF_E_UNSUPPORTED, "staged mode keeps no per-sample index maps on the device");
   switch (what) {
     case MF_EX_PERM: case MF_EX_BLOCKID: need = c->N; break;
     case MF_EX_RHO_R: need = c->m; break;

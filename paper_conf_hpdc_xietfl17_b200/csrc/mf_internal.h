@@ -15,6 +15,7 @@ constexpr int kMaxSegs = 8;  // blocks per Hogwild launch (a/G <= 8 strata block
 struct ChunkSegs {
   int64_t begin[kMaxSegs];
   int64_t prefix[kMaxSegs + 1];
+  int64_t shift[kMaxSegs];  // slot of chunk q = q*f + shift (0 resident; staged: buffer offset)
   int n;
 };
 
@@ -35,6 +36,7 @@ struct WavefrontLaunch {
   int storage, k, variant;  // variant 1 = ring-staged k_wavefront2 (needs dup), 0 = k_wavefront
   int lane_bytes;           // ring kernel: 16 (default) or 32 bytes per lane
   const Rating* slots;
+  int64_t shift;           // slot index offset (0 resident; staged: buffer offset - block start)
   const uint16_t* dup;     // per slot: distance to previous same-u (low byte) / same-v (high
                            // byte) sample of the sub-block if <= ring_window(), else 0
   const int64_t* sub_off;  // s*c + 1 slot offsets of this strata block's sub-blocks

@@ -50,7 +50,7 @@ __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slot
       int sgi = 0;
       while (ci >= segs.prefix[sgi + 1]) ++sgi;
       const uint32_t chunk = __ldg(chunks + segs.begin[sgi] + (ci - segs.prefix[sgi]));
-      lo = (int64_t)chunk * f;
+      lo = (int64_t)chunk * f + segs.shift[sgi];
     }
     // every group of the warp runs f iterations in lockstep (inactive ones on sentinels)
     run_serial<T, K, L, D, true>(slots, lo, f, act, P, Q, g, cp, cq, gl, gbase, 0xffffffffu);
@@ -101,7 +101,7 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
                                                    const int32_t* __restrict__ rank,
                                                    int* __restrict__ tickets, int s, int c,
                                                    T* __restrict__ P, T* __restrict__ Q, float g,
-                                                   float lp, float lq) {
+                                                   float lp, float lq, int64_t shift) {
   const int lane = threadIdx.x & 31;
   const int grp = lane / L, gl = lane % L, gbase = grp * L;
   const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
@@ -115,8 +115,8 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
     const int tgt = __ldg(my_rank + w);
     ticket_acquire(tickets + col, tgt);
     const int64_t sb = (int64_t)worker * c + col;
-    const int64_t lo = __ldg(sub_off + sb);
-    run_serial<T, K, L, 2, false>(slots, lo, (int)(__ldg(sub_off + sb + 1) - lo), true, P, Q, g, cp,
+    const int64_t lo = __ldg(sub_off + sb) + shift;
+    run_serial<T, K, L, 2, false>(slots, lo, (int)(__ldg(sub_off + sb + 1) + shift - lo), true, P, Q, g, cp,
                                   cq, gl, gbase, gmask);
     ticket_release(tickets + col, tgt + 1, gmask, gl);
   }
@@ -133,7 +133,7 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
                                                     const int32_t* __restrict__ rank,
                                                     int* __restrict__ tickets, int s, int c,
                                                     T* __restrict__ P, T* __restrict__ Q, float g,
-                                                    float lp, float lq) {
+                                                    float lp, float lq, int64_t shift) {
   extern __shared__ __align__(16) char smem[];
   constexpr int ROWB = K * (int)sizeof(T);
   const int lane = threadIdx.x & 31;
@@ -153,8 +153,8 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     const int col = __ldg(my_seq + w);
     const int tgt = __ldg(my_rank + w);
     const int64_t sb = (int64_t)worker * c + col;
-    const int64_t lo = __ldg(sub_off + sb);
-    const int n = (int)(__ldg(sub_off + sb + 1) - lo);
+    const int64_t lo = __ldg(sub_off + sb) + shift;
+    const int n = (int)(__ldg(sub_off + sb + 1) + shift - lo);
     ticket_acquire(tickets + col, tgt);     // (empty sub-blocks still keep the visit order)
     if (n > 0)
       run_subblock_ring<T, K, L, RS, F>(slots, dup, lo, n, P, Q, g, cp, cq, gl, gbase, gmask, ring);
@@ -270,7 +270,8 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
   T* P = reinterpret_cast<T*>(a.P);
   T* Q = reinterpret_cast<T*>(a.Q);
   float g = a.g, lp = a.lp, lq = a.lq;
-  void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq};
+  int64_t shift = a.shift;
+  void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq, &shift};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, 0,
                                      a.stream);
 }
@@ -305,7 +306,9 @@ static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
   T* P = reinterpret_cast<T*>(a.P);
   T* Q = reinterpret_cast<T*>(a.Q);
   float g = a.g, lp = a.lp, lq = a.lq;
-  void* args[] = {&slots, &dup, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq};
+  int64_t shift = a.shift;
+  void* args[] = {&slots, &dup, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq,
+                  &shift};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, smem,
                                      a.stream);
 }

@@ -48,7 +48,7 @@ class Params(ctypes.Structure):
                 ("batch_f", ctypes.c_int32), ("wf_cols", ctypes.c_int32),
                 ("grid_a", ctypes.c_int32), ("cyclic", ctypes.c_int32),
                 ("lane_bytes", ctypes.c_int32), ("prefetch", ctypes.c_int32),
-                ("wf_kernel", ctypes.c_int32),
+                ("staged", ctypes.c_int32), ("wf_kernel", ctypes.c_int32),
                 ("device", ctypes.c_int32),
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("transport", ctypes.c_int32), ("nccl_id", ctypes.c_void_p),
@@ -182,7 +182,8 @@ class MF:
                  init_scale: float = 1.0, rating_scale: float = 1.0, seed: int = 42,
                  schedule: str = "hogwild", storage: str = "fp32", workers: int = 0,
                  batch_f: int = 256, wf_cols: int = 0, grid_a: int = 0, cyclic: bool = False,
-                 lane_bytes: int = 0, prefetch: int = 0, wf_kernel: int = 0, device: int = 0, rank: int = 0, world: int = 1,
+                 lane_bytes: int = 0, prefetch: int = 0, wf_kernel: int = 0, staged: bool = False,
+                 device: int = 0, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, transport: int = 0, stream=None,
                  allocator: str = "torch"):
         L = lib()
@@ -196,6 +197,7 @@ class MF:
         p.schedule, p.storage = SCHEDULE[schedule], STORAGE[storage]
         p.workers, p.batch_f, p.wf_cols, p.grid_a = workers, batch_f, wf_cols, grid_a
         p.cyclic, p.lane_bytes, p.prefetch, p.wf_kernel = int(cyclic), lane_bytes, prefetch, wf_kernel
+        p.staged = int(staged)
         p.device, p.rank, p.world, p.transport = device, rank, world, transport
         self._id_buf = None
         if nccl_id is not None:

@@ -56,12 +56,13 @@ def run_ranks(world, R, k, epochs, **kw):
 
 @pytest.mark.parametrize("world", [2, 4])
 @pytest.mark.parametrize("kw", [dict(schedule="wavefront", workers=4, wf_cols=5),
-                                dict(schedule="hogwild", workers=1, batch_f=64)])
+                                dict(schedule="hogwild", workers=1, batch_f=64),
+                                dict(schedule="wavefront", workers=4, wf_cols=5, staged=True)])
 def test_multirank_strata_matches_oracle(world, kw):
     R = synth.tiny(seed=0)
     epochs = 2
     res = run_ranks(world, R, 16, epochs, **kw)
-    okw = {k: v for k, v in kw.items()}
+    okw = {k: v for k, v in kw.items() if k != "staged"}
     o = po.Oracle(R.m, R.n, 16, R.u, R.v, R.r, grid_a=8, **HP, **okw)
     for _ in range(epochs):
         o.train_epoch()

@@ -294,3 +294,31 @@ def test_checkpoint_resume_equals_uninterrupted(tiny):
     c.train_epoch()
     c.train_epoch()
     assert np.array_equal(a.factors()[0], c.factors()[0])
+
+
+# ----------------------------------------------------------------------------- out-of-core
+
+@pytest.mark.parametrize("kw", [dict(schedule="wavefront", workers=4, wf_cols=5, grid_a=8),
+                                dict(schedule="wavefront", workers=4, wf_cols=5, grid_a=1),
+                                dict(schedule="hogwild", workers=1, grid_a=8, batch_f=64),
+                                dict(schedule="wavefront", workers=6, wf_cols=9, grid_a=4, k=128)])
+def test_staged_equals_resident(kw):
+    """Section 6.2 out-of-core mode: ratings in pinned host memory, streamed per stratum through
+    two HBM buffers (copy stream overlapping compute, also across epochs).  Same order, so the
+    deterministic result is bit-identical to the resident run."""
+    kw = dict(kw)
+    k = kw.pop("k", 32)
+    R = ragged()
+    out = []
+    for staged in (False, True):
+        g = mf.MF(R.m, R.n, k, staged=staged, **TABLE3_NETFLIX, **kw)
+        g.load(R.u, R.v, R.r)
+        g.load(R.ut, R.vt, R.rt, "test")
+        for _ in range(3):
+            g.train_epoch()
+        out.append((g.factors(), g.rmse()))
+        g.close()
+    (P0, Q0), r0 = out[0]
+    (P1, Q1), r1 = out[1]
+    assert np.array_equal(P0, P1) and np.array_equal(Q0, Q1)
+    assert r0 == r1
