@@ -1237,6 +1237,9 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
       ++segs.n;
     }
     if (segs.n == 0) return MF_OK;
+    segs.minlen = segs.prefix[1] - segs.prefix[0];
+    for (int s2 = 1; s2 < segs.n; ++s2)
+      segs.minlen = std::min(segs.minlen, segs.prefix[s2 + 1] - segs.prefix[s2]);
     CUDA_TRY(c, cudaMemsetAsync(c->counter, 0, sizeof(unsigned long long), c->st));
     HogwildLaunch L{};
     L.storage = c->p.storage; L.k = c->k; L.lane_bytes = c->p.lane_bytes ? c->p.lane_bytes : 16;

@@ -16,6 +16,7 @@ struct ChunkSegs {
   int64_t begin[kMaxSegs];
   int64_t prefix[kMaxSegs + 1];
   int64_t shift[kMaxSegs];  // slot of chunk q = q*f + shift (0 resident; staged: buffer offset)
+  int64_t minlen;           // shortest segment (chunks): claims interleave the segments
   int n;
 };
 
