@@ -48,6 +48,8 @@ def parse():
     ap.add_argument("--staged", action="store_true",
                     help="out-of-core: ratings in pinned host memory, streamed per stratum")
     ap.add_argument("--grid-a", type=int, default=0)
+    ap.add_argument("--batch-f", type=int, default=0,
+                    help="Eq. 8 f (0 = 256 on 1 GPU, 1024 with strata; DESIGN.md section 7)")
     ap.add_argument("--fraction", type=float, default=1.0, help="scale the workload (testing)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -211,7 +213,8 @@ def run_reference(args):
 def config_of(args, R):
     return {"workload": f"{args.workload}-shaped synthetic (Table 2 shape, power-law skew)",
             "m": R.m, "n": R.n, "N_train": R.N, "N_test": R.Ntest, "k": args.k,
-            "storage": args.storage, "schedule": args.schedule, "batch_f": 256,
+            "storage": args.storage, "schedule": args.schedule,
+            "batch_f": args.batch_f or (1024 if args.gpus > 1 or args.grid_a > 1 else 256),
             "parallelism": f"dsgd-strata{args.gpus}" if args.gpus > 1 else "1gpu",
             "staged": bool(args.staged), "grid_a": args.grid_a or (8 if args.gpus > 1 else 1),
             "l2": "inputs larger than L2 (COO %.2f GB per epoch); model P+Q stays cached as in "
@@ -235,7 +238,8 @@ def main():
         nccl_id = mf.nccl_unique_id_via()
     kw = dict(schedule=args.schedule, storage=args.storage, workers=args.workers,
               wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes, prefetch=args.prefetch,
-              wf_kernel=args.wf_kernel, staged=args.staged, grid_a=args.grid_a, seed=42,
+              wf_kernel=args.wf_kernel, staged=args.staged, grid_a=args.grid_a,
+              batch_f=args.batch_f or (1024 if world > 1 or args.grid_a > 1 else 256), seed=42,
               device=local, rank=rank, world=world, nccl_id=nccl_id, **hp)
     torch.cuda.synchronize()
     model = mf.MF(R.m, R.n, args.k, stream=stream, **kw)

@@ -48,6 +48,28 @@ __global__ void k_iota_keys(uint64_t S, int64_t n, uint64_t* __restrict__ keys,
   }
 }
 
+// keys[j] = key(S, idx[j]) (idx == nullptr: idx[j] = j), vals[j] = idx[j]
+__global__ void k_keys_of(uint64_t S, const uint32_t* __restrict__ idx, int64_t n,
+                          uint64_t* __restrict__ keys, uint32_t* __restrict__ vals) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t i = idx ? idx[j] : (uint32_t)j;
+    keys[j] = hkey(S, (uint64_t)i);
+    vals[j] = i;
+  }
+}
+
+// world > 1: flag the caller's ratings whose row segment this rank owns
+__global__ void k_own_caller(const int32_t* __restrict__ u, int64_t N, const int32_t* __restrict__ rho_r,
+                             int64_t m, int64_t a, int64_t lo_seg, int64_t hi_seg,
+                             char* __restrict__ flag) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = (int64_t)rho_r[u[i]] * a / m;
+    flag[i] = (r >= lo_seg && r < hi_seg) ? 1 : 0;
+  }
+}
+
 // rho[perm[j]] = j
 __global__ void k_rank_of(const uint32_t* __restrict__ perm, int64_t n, int32_t* __restrict__ rho) {
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n;
@@ -927,9 +949,36 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
   float* orr;
   TRY(stage_input(c, N, u, v, r, on_device, &du, &dv, &dr, &ou, &ov, &orr));
   TRY(validate(c, N, du, dv, dr));
+
+  // relabel (A: S_ROW, S_COL) first: a rank only needs the ratings of the row segments it owns
+  TRY(relabel(c, kTagRow, c->m, &c->rho_r));
+  TRY(relabel(c, kTagCol, c->n, &c->rho_c));
+  uint32_t* own = nullptr;                  // caller indices of this rank's ratings (world > 1)
+  if (c->G > 1 && N > 0) {
+    char* flag = nullptr;
+    int64_t* nsel = nullptr;
+    TRY(c->alloc(&flag, (size_t)N));
+    TRY(c->alloc(&own, (size_t)N));
+    TRY(c->alloc(&nsel, 1));
+    k_own_caller<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(du, N, c->rho_r, c->m, c->a,
+                                                             c->lo_row_seg(), c->hi_row_seg(), flag);
+    KERNEL_TRY(c);
+    cub::CountingInputIterator<uint32_t> iota(0);
+    size_t bytes = 0;
+    CUDA_TRY(c, cub::DeviceSelect::Flagged(nullptr, bytes, iota, flag, own, nsel, N, c->st));
+    TRY(c->need_tmp(bytes));
+    CUDA_TRY(c, cub::DeviceSelect::Flagged(c->tmp, bytes, iota, flag, own, nsel, N, c->st));
+    int64_t h = 0;
+    CUDA_TRY(c, cudaMemcpyAsync(&h, nsel, 8, cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    c->release(flag);
+    c->release(nsel);
+    N = h;
+  }
   c->N = N;
 
-  // Alg. 1 l.2 random_shuffle: storage order = perm(S_SHUF, N)
+  // Alg. 1 l.2 random_shuffle: storage order = perm(S_SHUF, N) over caller indices.
+  // A rank sorts only its own ratings by the same keys: their relative order is the global one.
   {
     uint64_t *k0 = nullptr, *k1 = nullptr;
     uint32_t* v0 = nullptr;
@@ -938,16 +987,14 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
     TRY(c->alloc(&v0, (size_t)N));
     TRY(c->alloc(&c->perm, (size_t)N));
     if (N > 0) {
-      k_iota_keys<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(
-          make_stream(c->p.seed, kTagShuf, 0, 0), N, k0, v0);
+      k_keys_of<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(make_stream(c->p.seed, kTagShuf, 0, 0),
+                                                           own, N, k0, v0);
       KERNEL_TRY(c);
       TRY(c->sort_pairs(k0, k1, v0, c->perm, N, 64));
     }
     c->release(k0); c->release(k1); c->release(v0);
+    c->release(own);
   }
-  // relabel (A: S_ROW, S_COL)
-  TRY(relabel(c, kTagRow, c->m, &c->rho_r));
-  TRY(relabel(c, kTagCol, c->n, &c->rho_c));
 
   // storage-order samples (relabelled, scaled) and their buckets
   Grid Gd{c->m, c->n, c->a, c->s, c->c, c->wf};
