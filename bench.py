@@ -232,6 +232,8 @@ def main():
     from paper_conf_hpdc_xietfl17_b200 import mf
 
     R, hp = workload(args, device)
+    if R.N > (1 << 30):       # Hugewiki-shaped: no second copy of the set for e2e / extra runs
+        args.no_e2e = args.no_cpu_baseline = args.no_deterministic = True
     stream = torch.cuda.Stream(device=device)
     nccl_id = None
     if world > 1:

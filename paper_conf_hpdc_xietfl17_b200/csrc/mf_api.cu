@@ -1013,6 +1013,8 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
     KERNEL_TRY(c);
   }
   c->release(ou); c->release(ov); c->release(orr);
+  const bool keep_maps = N <= ((int64_t)1 << 30);   // per-sample index maps only feed exports
+  if (!keep_maps) c->release(c->perm);
 
   // bucket counts -> offsets
   unsigned int* cnt = nullptr;
@@ -1079,11 +1081,20 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
     CUDA_TRY(c, cudaMemcpyAsync(c->d_choff, c->ch_off.data(), (nb + 1) * 8, cudaMemcpyHostToDevice, c->st));
     CUDA_TRY(c, cudaStreamSynchronize(c->st));  // host vectors used by async copies
   }
+  // free the bucket sort's inputs before the slot array (peak HBM at Hugewiki scale)
+  if (keys_sorted) {
+    c->release(bk0);
+    c->release(pos0);
+  } else {
+    c->release(bk0);
+    c->release(bk1);
+    c->release(pos1);
+  }
   TRY(c->alloc(&c->slots, (size_t)std::max<int64_t>(c->nslots, 1)));
-  TRY(c->alloc(&c->slot_pos, (size_t)std::max<int64_t>(c->nslots, 1)));
+  if (keep_maps) TRY(c->alloc(&c->slot_pos, (size_t)std::max<int64_t>(c->nslots, 1)));
   if (c->nslots > N) {
     CUDA_TRY(c, cudaMemsetAsync(c->slots, 0xFF, c->nslots * sizeof(Rating), c->st));  // u=v=-1
-    CUDA_TRY(c, cudaMemsetAsync(c->slot_pos, 0xFF, c->nslots * 4, c->st));
+    if (c->slot_pos) CUDA_TRY(c, cudaMemsetAsync(c->slot_pos, 0xFF, c->nslots * 4, c->st));
   }
   if (N > 0) {
     k_place<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(
@@ -1616,8 +1627,8 @@ mf_status mf_export_schedule(mf_ctx* c, int32_t what, int32_t epoch, int64_t* bu
   if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
   const int64_t nb = (int64_t)c->a * c->a;
   int64_t need = 0;
-  if (c->staged && (what == MF_EX_PERM || what == MF_EX_BLOCKID))
-    return c->fail(MF_E_UNSUPPORTED, "staged mode keeps no per-sample index maps on the device");
+  if ((what == MF_EX_PERM && !c->perm) || (what == MF_EX_BLOCKID && !c->slot_pos))
+    return c->fail(MF_E_UNSUPPORTED, "per-sample index maps are not kept (staged mode or N > 2^30)");
   switch (what) {
     case MF_EX_PERM: case MF_EX_BLOCKID: need = c->N; break;
     case MF_EX_RHO_R: need = c->m; break;
