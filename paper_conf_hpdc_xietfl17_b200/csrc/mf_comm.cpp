@@ -4,6 +4,7 @@
 #include <dlfcn.h>
 #include <nccl.h>
 
+#include <chrono>
 #include <condition_variable>
 #include <cstring>
 #include <map>
@@ -80,22 +81,36 @@ struct LoopGroup {
   std::vector<cudaEvent_t> ev;                 // each rank's "my stream reached here" event
   std::vector<std::vector<void*>> ptrs;        // published device pointers per rank
 
-  void barrier() {
+  // Returns false if the other ranks do not arrive within 300 s (a rank failed mid-protocol);
+  // the group is then poisoned so every later barrier fails fast instead of hanging.
+  bool barrier() {
     std::unique_lock<std::mutex> l(mu);
+    if (broken) return false;
     const uint64_t g = gen;
     if (++arrived == world) {
       arrived = 0;
       ++gen;
       cv.notify_all();
-    } else {
-      cv.wait(l, [&] { return gen != g; });
+      return true;
     }
+    if (!cv.wait_for(l, std::chrono::seconds(300), [&] { return gen != g || broken; }) || broken) {
+      broken = true;
+      cv.notify_all();
+      return false;
+    }
+    return true;
   }
+  bool broken = false;
 };
 
 namespace {
 std::mutex g_reg_mu;
 std::map<std::string, std::shared_ptr<LoopGroup>> g_reg;
+
+bool lb_fail(std::string* why) {
+  if (why) *why = "loopback: a rank did not reach the rendezvous (timeout or earlier failure)";
+  return false;
+}
 
 bool cuda_ok(cudaError_t e, const char* what, std::string* why) {
   if (e == cudaSuccess) return true;
@@ -134,7 +149,11 @@ Comm* Comm::create_loopback(const uint8_t id[128], int world, int rank, cudaStre
     return nullptr;
   }
   g->ev[(size_t)rank] = c->ev_;
-  g->barrier();                                // all ranks joined (like ncclCommInitRank)
+  if (!g->barrier()) {                         // all ranks joined (like ncclCommInitRank)
+    if (why) *why = "loopback: not every rank joined within the timeout";
+    destroy(c);
+    return nullptr;
+  }
   return c;
 }
 
@@ -180,7 +199,7 @@ bool Comm::exchange(const std::vector<Xfer>& xs, int me, std::string* why) {
     for (const Xfer& x : xs) mine.push_back(x.ptr);
     g.ptrs[(size_t)me] = mine;
     if (!cuda_ok(cudaEventRecord(ev_, st_), "cudaEventRecord", why)) return false;
-    g.barrier();                               // every rank's segments are final on its stream
+    if (!g.barrier()) return lb_fail(why);         // every rank's segments are final on its stream
     for (size_t i = 0; i < xs.size(); ++i)
       if (xs[i].dst == me) {
         if (!cuda_ok(cudaStreamWaitEvent(st_, g.ev[(size_t)xs[i].src], 0), "wait", why)) return false;
@@ -188,13 +207,13 @@ bool Comm::exchange(const std::vector<Xfer>& xs, int me, std::string* why) {
                                      cudaMemcpyDeviceToDevice, st_), "copy", why))
           return false;
       }
-    g.barrier();                               // all copies enqueued before events are re-recorded
+    if (!g.barrier()) return lb_fail(why);         // all copies enqueued before events are re-recorded
     if (!cuda_ok(cudaEventRecord(ev_, st_), "cudaEventRecord", why)) return false;
-    g.barrier();
+    if (!g.barrier()) return lb_fail(why);
     for (size_t i = 0; i < xs.size(); ++i)     // a source does not overwrite before the copy ran
       if (xs[i].src == me && !cuda_ok(cudaStreamWaitEvent(st_, g.ev[(size_t)xs[i].dst], 0), "wait", why))
         return false;
-    g.barrier();
+    if (!g.barrier()) return lb_fail(why);
     return true;
   }
   Nccl* L = nccl(why);
@@ -228,7 +247,7 @@ bool Comm::allreduce_sum(double* dptr, size_t n, std::string* why) {
     LoopGroup& g = *loop_;
     g.ptrs[(size_t)rank_] = {dptr};
     if (!cuda_ok(cudaEventRecord(ev_, st_), "cudaEventRecord", why)) return false;
-    g.barrier();
+    if (!g.barrier()) return lb_fail(why);
     std::vector<double> acc(n, 0.0), tmp(n);
     for (int r = 0; r < world_; ++r) {         // fixed rank order: identical sum on every rank
       if (!cuda_ok(cudaStreamWaitEvent(st_, g.ev[(size_t)r], 0), "wait", why)) return false;
@@ -238,12 +257,12 @@ bool Comm::allreduce_sum(double* dptr, size_t n, std::string* why) {
         return false;
       for (size_t i = 0; i < n; ++i) acc[i] += tmp[i];
     }
-    g.barrier();                               // everyone read every input before overwriting
+    if (!g.barrier()) return lb_fail(why);         // everyone read every input before overwriting
     if (!cuda_ok(cudaMemcpyAsync(dptr, acc.data(), n * sizeof(double), cudaMemcpyHostToDevice, st_),
                  "copy", why) ||
         !cuda_ok(cudaStreamSynchronize(st_), "sync", why))
       return false;
-    g.barrier();
+    if (!g.barrier()) return lb_fail(why);
     return true;
   }
   Nccl* L = nccl(why);
