@@ -82,7 +82,8 @@ typedef struct mf_params {
                              wavefront = row sub-blocks per strata block (0 = min(768, m/(4a)))             */
   int32_t batch_f;        /* Eq. 8 batch f (0 = 256)                                    */
   int32_t wf_cols;        /* wavefront column sub-blocks c (0 = 2*s, R9)                        */
-  int32_t grid_a;         /* strata grid a x a (0 = 1 if world == 1 else 8); a % world == 0      */
+  int32_t grid_a;         /* strata grid a x a (0 = 1 if world == 1 else 8); a % world == 0
+                             and a / world <= 16                                                */
   int32_t cyclic;         /* wavefront: 1 = cyclic column order (A: cyclic variant), needs c >= s */
   int32_t lane_bytes;     /* Hogwild/RMSE kernel: bytes of p_u (and q_v) per lane, 16 or 32 (0 = 16) */
   int32_t prefetch;       /* Hogwild software-pipeline depth: samples in flight per worker, 1 or 2 (0 = 1) */

@@ -660,7 +660,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
   const int a = p->grid_a > 0 ? p->grid_a : (world == 1 ? 1 : 8);
-  if (a % world != 0 || a > p->m || a > p->n || a > 64) return MF_E_INVAL;
+  if (a % world != 0 || a > p->m || a > p->n || a > 64 || a / world > kMaxSegs) return MF_E_INVAL;
   if (p->batch_f < 0 || p->workers < 0 || p->wf_cols < 0) return MF_E_INVAL;
 
   mf_ctx* c = new (std::nothrow) mf_ctx();

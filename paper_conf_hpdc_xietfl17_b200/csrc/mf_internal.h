@@ -9,7 +9,7 @@
 
 namespace mfb {
 
-constexpr int kMaxSegs = 8;  // blocks per Hogwild launch (a/G <= 8 strata blocks)
+constexpr int kMaxSegs = 16;  // blocks per Hogwild launch: a/G <= 16 (checked by mf_create)
 
 // Chunk list of one Hogwild launch: segment s is chunks[begin[s] .. begin[s] + prefix[s+1]-prefix[s]).
 struct ChunkSegs {
