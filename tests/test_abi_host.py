@@ -59,6 +59,8 @@ def test_create_rejects_bad_params_before_touching_a_device(L):
     p.storage = 0
     p.world, p.grid_a = 3, 8                                         # a % world != 0
     assert L.mf_create(ctypes.byref(p), ctypes.byref(h)) == -1
+    p.world, p.grid_a = 1, 32                                        # a / world > 16 blocks
+    assert L.mf_create(ctypes.byref(p), ctypes.byref(h)) == -1
     bad = mf.Params()
     assert L.mf_create(ctypes.byref(bad), ctypes.byref(h)) == -1     # struct_size unset
     assert not h.value
