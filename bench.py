@@ -37,7 +37,7 @@ def parse():
     ap.add_argument("--impl", default="mf", choices=["mf", "reference"])
     ap.add_argument("--workload", default="netflix", choices=["netflix", "yahoo", "hugewiki", "tiny"])
     ap.add_argument("--storage", default="fp16", choices=["fp16", "fp32", "bf16"])
-    ap.add_argument("--schedule", default="hogwild", choices=["hogwild", "wavefront"])
+    ap.add_argument("--schedule", default="hogwild", choices=["hogwild", "wavefront", "libmf"])
     ap.add_argument("--k", type=int, default=128)
     ap.add_argument("--workers", type=int, default=0)
     ap.add_argument("--wf-cols", type=int, default=0)

@@ -56,7 +56,13 @@ enum {
 };
 
 typedef enum { MF_FP32 = 0, MF_FP16 = 1, MF_BF16 = 2 } mf_storage;   /* P:L242 feature storage */
-typedef enum { MF_HOGWILD = 0, MF_WAVEFRONT = 1 } mf_schedule;      /* section 5.1 / 5.2 */
+typedef enum {
+  MF_HOGWILD = 0,   /* batch-Hogwild! (section 5.1)                                           */
+  MF_WAVEFRONT = 1, /* deterministic wavefront (section 5.2)                                  */
+  MF_LIBMF = 2      /* BASELINE: LIBMF-GPU global-table block scheduler (section 5, Fig. 5a,
+                       P:L258-268); grid_a x grid_a blocks (0 = 64), workers = warps (0 = a/2);
+                       one GPU, resident ratings only                                          */
+} mf_schedule;
 typedef enum { MF_TRAIN = 0, MF_TEST = 1 } mf_set;
 
 /* Device-memory hooks (e.g. torch's caching allocator).  alloc returns NULL on failure. */

@@ -446,6 +446,10 @@ struct mf_ctx {
   // out-of-core staging (params.staged; section 6.2): the bucketed ratings live in
   // pinned host memory; each stratum's blocks are copied into one of two device buffers on a
   // copy stream while the previous stratum computes.
+  bool libmf = false;              // LIBMF-GPU table-scheduler baseline (MF_LIBMF)
+  int64_t *d_blk_off = nullptr, *d_blk_len = nullptr;
+  int *lm_lock = nullptr, *lm_row = nullptr, *lm_col = nullptr, *lm_done = nullptr, *lm_rem = nullptr;
+
   bool staged = false;
   Rating* h_slots = nullptr;
   uint16_t* h_dup = nullptr;
@@ -648,7 +652,9 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->m <= 0 || p->n <= 0 || p->m >= INT32_MAX || p->n >= INT32_MAX) return MF_E_INVAL;
   if (!(p->k == 16 || p->k == 32 || p->k == 64 || p->k == 128 || p->k == 256))
     return MF_E_UNSUPPORTED;
-  if (p->storage < 0 || p->storage > 2 || p->schedule < 0 || p->schedule > 1) return MF_E_INVAL;
+  if (p->storage < 0 || p->storage > 2 || p->schedule < 0 || p->schedule > 2) return MF_E_INVAL;
+  const bool libmf = p->schedule == MF_LIBMF;
+  if (libmf && (p->world > 1 || p->staged)) return MF_E_UNSUPPORTED;
   if (!(p->alpha >= 0.f) || !(p->beta >= 0.f) || !(p->lambda_p >= 0.f) || !(p->lambda_q >= 0.f))
     return MF_E_INVAL;
   if (!(p->rating_scale > 0.f) || !(p->init_scale > 0.f)) return MF_E_INVAL;
@@ -659,8 +665,10 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->staged < 0 || p->staged > 1) return MF_E_INVAL;
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
-  const int a = p->grid_a > 0 ? p->grid_a : (world == 1 ? 1 : 8);
-  if (a % world != 0 || a > p->m || a > p->n || a > 64 || a / world > kMaxSegs) return MF_E_INVAL;
+  const int a = p->grid_a > 0 ? p->grid_a : (libmf ? 64 : (world == 1 ? 1 : 8));
+  if (a % world != 0 || a > p->m || a > p->n) return MF_E_INVAL;
+  if (!libmf && (a > 64 || a / world > kMaxSegs)) return MF_E_INVAL;
+  if (libmf && a > 1024) return MF_E_INVAL;
   if (p->batch_f < 0 || p->workers < 0 || p->wf_cols < 0) return MF_E_INVAL;
 
   mf_ctx* c = new (std::nothrow) mf_ctx();
@@ -675,6 +683,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   c->rank = p->rank;
   c->f = p->batch_f > 0 ? p->batch_f : 256;
   c->wf = p->schedule == MF_WAVEFRONT;
+  c->libmf = p->schedule == MF_LIBMF;
   c->staged = p->staged == 1;
   if (c->wf) {
     const int64_t rows_per_seg = p->m / a;
@@ -1079,6 +1088,17 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
     CUDA_TRY(c, cudaMemcpyAsync(dst_off, c->blk_off.data(), (nb + 1) * 8, cudaMemcpyHostToDevice, c->st));
     TRY(c->alloc(&c->d_choff, (size_t)nb + 1));
     CUDA_TRY(c, cudaMemcpyAsync(c->d_choff, c->ch_off.data(), (nb + 1) * 8, cudaMemcpyHostToDevice, c->st));
+    if (c->libmf) {
+      TRY(c->alloc(&c->d_blk_off, (size_t)nb + 1));
+      TRY(c->alloc(&c->d_blk_len, (size_t)nb));
+      TRY(c->alloc(&c->lm_lock, 1));
+      TRY(c->alloc(&c->lm_rem, 1));
+      TRY(c->alloc(&c->lm_row, (size_t)c->a));
+      TRY(c->alloc(&c->lm_col, (size_t)c->a));
+      TRY(c->alloc(&c->lm_done, (size_t)nb));
+      CUDA_TRY(c, cudaMemcpyAsync(c->d_blk_off, c->blk_off.data(), (nb + 1) * 8, cudaMemcpyHostToDevice, c->st));
+      CUDA_TRY(c, cudaMemcpyAsync(c->d_blk_len, c->blk_len.data(), nb * 8, cudaMemcpyHostToDevice, c->st));
+    }
     CUDA_TRY(c, cudaStreamSynchronize(c->st));  // host vectors used by async copies
   }
   // free the bucket sort's inputs before the slot array (peak HBM at Hugewiki scale)
@@ -1189,6 +1209,7 @@ mf_status mf_load_coo(mf_ctx* c, int32_t set, int64_t nnz, const int32_t* u, con
 // ---------------------------------------------------------------------------------------------
 static mf_status build_schedule(mf_ctx* c, int32_t t) {
   const int64_t nb = (int64_t)c->a * c->a;
+  if (c->libmf) return MF_OK;             // blocks are picked at run time from the table
   if (!c->wf) {
     const int64_t total = c->ch_off.back();
     if (total == 0) return MF_OK;
@@ -1406,6 +1427,37 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   CUDA_TRY(c, cudaEventRecord(c->ev_s0, c->st));
   TRY(build_schedule(c, t));
   CUDA_TRY(c, cudaEventRecord(c->ev_s1, c->st));
+  if (c->libmf) {
+    const int64_t nb = (int64_t)c->a * c->a;
+    const int rem = (int)nb;
+    CUDA_TRY(c, cudaMemsetAsync(c->lm_lock, 0, 4, c->st));
+    CUDA_TRY(c, cudaMemsetAsync(c->lm_row, 0, (size_t)c->a * 4, c->st));
+    CUDA_TRY(c, cudaMemsetAsync(c->lm_col, 0, (size_t)c->a * 4, c->st));
+    CUDA_TRY(c, cudaMemsetAsync(c->lm_done, 0, (size_t)nb * 4, c->st));
+    CUDA_TRY(c, cudaMemcpyAsync(c->lm_rem, &rem, 4, cudaMemcpyHostToDevice, c->st));
+    LibmfLaunch L{};
+    L.storage = c->p.storage; L.k = c->k; L.slots = c->slots; L.blk_off = c->d_blk_off;
+    L.blk_len = c->d_blk_len; L.a = c->a; L.lock = c->lm_lock; L.row_busy = c->lm_row;
+    L.col_busy = c->lm_col; L.done = c->lm_done; L.remaining = c->lm_rem;
+    L.workers = c->p.workers > 0 ? c->p.workers : std::max(1, c->a / 2);
+    L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q;
+    L.seed = make_stream(c->p.seed, 11, (uint64_t)t, 0); L.stream = c->st; L.out_lanes = &c->last_lanes;
+    CUDA_TRY(c, cudaEventRecord(ev_at(c, 0), c->st));
+    CUDA_TRY(c, launch_libmf(L));
+    CUDA_TRY(c, cudaEventRecord(ev_at(c, 1), c->st));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));   // the host-side copy of `rem` must outlive it
+    c->n_sgd = 1;
+    c->n_launch += 1;
+    c->updates = c->N;
+    c->last_workers = L.workers;
+    c->last_grid = L.workers;
+    c->last_block = 32;
+    CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
+    c->t = t + 1;
+    c->have_stats = true;
+    if (epoch_done) *epoch_done = c->t;
+    return MF_OK;
+  }
   // holders of every Q segment's valid copy persist across sub-epochs and epochs (comm);
   // world == 1 keeps a local vector (every segment is always on rank 0: no transfers)
   std::vector<int32_t> local_hold((size_t)c->a, -1);

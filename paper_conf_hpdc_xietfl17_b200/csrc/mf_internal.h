@@ -62,7 +62,22 @@ struct RmseLaunch {
   cudaStream_t stream;
 };
 
+struct LibmfLaunch {
+  int storage, k;
+  const Rating* slots;
+  const int64_t *blk_off, *blk_len;  // a*a padded block starts / sample counts
+  int a;
+  int *lock, *row_busy, *col_busy, *done, *remaining;
+  int workers;
+  void *P, *Q;
+  float g, lp, lq;
+  uint64_t seed;
+  cudaStream_t stream;
+  int* out_lanes;
+};
+
 cudaError_t launch_hogwild(const HogwildLaunch& a);
+cudaError_t launch_libmf(const LibmfLaunch& a);
 cudaError_t launch_wavefront(const WavefrontLaunch& a);
 cudaError_t launch_rmse(const RmseLaunch& a);
 int ring_window(int k, int storage);  // history window W of k_wavefront2 for this geometry

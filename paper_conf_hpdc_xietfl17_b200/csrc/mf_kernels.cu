@@ -162,6 +162,82 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
   }
 }
 
+
+// ---------------------------------------------------------------------------------------------
+// LIBMF-GPU table scheduler (paper section 5, Fig. 5a): the in-tree BASELINE the
+// paper's schedulers replace.  R is cut into a x a blocks; a worker (one warp, L active lanes)
+// takes the single global lock, scans the table for a block whose row and column are free and
+// which has not been updated this epoch (random start, then O(a^2) worst case), marks its row
+// and column busy, releases the lock, updates the block serially, and frees its row/column.
+// Conflict-free (serialisable) but nondeterministic order; every block once per epoch.
+// ---------------------------------------------------------------------------------------------
+template <typename T, int K, int L>
+__global__ void __launch_bounds__(32) k_libmf(const Rating* __restrict__ slots,
+                                              const int64_t* __restrict__ blk_off,
+                                              const int64_t* __restrict__ blk_len, int a,
+                                              int* lock, int* row_busy, int* col_busy, int* done,
+                                              int* remaining, int workers, T* __restrict__ P,
+                                              T* __restrict__ Q, float g, float lp, float lq,
+                                              uint64_t seed) {
+  const int lane = threadIdx.x & 31;
+  if (lane >= L) return;
+  const int worker = blockIdx.x;
+  if (worker >= workers) return;
+  const unsigned gmask = (L == 32) ? 0xffffffffu : ((1u << L) - 1u);
+  const float cp = 1.f - g * lp, cq = 1.f - g * lq;
+  uint64_t draw = mix64(seed + (uint64_t)worker * kPhi);
+  unsigned ns = 64;
+  for (;;) {
+    int b = -1;
+    if (lane == 0) {
+      while (atomicCAS(lock, 0, 1) != 0) __nanosleep(64);
+      __threadfence();
+      if (*(volatile int*)remaining == 0) {
+        b = -2;
+      } else {
+        draw = mix64(draw + kPhi);
+        const int r0 = (int)(draw % (uint64_t)a), c0 = (int)((draw >> 32) % (uint64_t)a);
+        for (int dr = 0; dr < a && b < 0; ++dr) {
+          const int r = (r0 + dr) % a;
+          if (((volatile int*)row_busy)[r]) continue;
+          for (int dc = 0; dc < a; ++dc) {
+            const int cc = (c0 + dc) % a;
+            if (!((volatile int*)col_busy)[cc] && !((volatile int*)done)[r * a + cc]) {
+              b = r * a + cc;
+              break;
+            }
+          }
+        }
+        if (b >= 0) {
+          row_busy[b / a] = 1;
+          col_busy[b % a] = 1;
+          done[b] = 1;
+          *remaining -= 1;
+        }
+      }
+      __threadfence();
+      atomicExch(lock, 0);
+    }
+    b = __shfl_sync(gmask, b, 0);
+    if (b == -2) break;
+    if (b == -1) {                        // nothing independent is free: back off and retry
+      __nanosleep(ns);
+      if (ns < 4096) ns <<= 1;
+      continue;
+    }
+    ns = 64;
+    const int64_t lo = __ldg(blk_off + b);
+    run_serial<T, K, L, 1, false>(slots, lo, (int)__ldg(blk_len + b), true, P, Q, g, cp, cq, lane, 0,
+                                  gmask);
+    __threadfence();
+    __syncwarp(gmask);
+    if (lane == 0) {
+      atomicExch(row_busy + b / a, 0);
+      atomicExch(col_busy + b % a, 0);
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------------------------
 // RMSE (R13): per-group fp32 dot, per-lane-0 fp64 accumulation, fixed-order block
 // reduction to one partial per CTA; k_rmse_final sums the partials in a fixed order.
@@ -314,6 +390,15 @@ static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
 }
 
 template <typename T, int K, int L>
+static cudaError_t launch_libmf_t(const LibmfLaunch& a) {
+  if (a.out_lanes) *a.out_lanes = L;
+  k_libmf<T, K, L><<<a.workers, 32, 0, a.stream>>>(
+      a.slots, a.blk_off, a.blk_len, a.a, a.lock, a.row_busy, a.col_busy, a.done, a.remaining,
+      a.workers, reinterpret_cast<T*>(a.P), reinterpret_cast<T*>(a.Q), a.g, a.lp, a.lq, a.seed);
+  return cudaGetLastError();
+}
+
+template <typename T, int K, int L>
 static cudaError_t launch_rmse_t(const RmseLaunch& a) {
   const int threads = 256;
   const int blocks = a.num_sms * 4;
@@ -341,6 +426,11 @@ template <typename T, int K>
 static cudaError_t hogwild_k(const HogwildLaunch& a) {
   if (a.lane_bytes == 32) return hogwild_kl<T, K, 32>(a);
   return hogwild_kl<T, K, 16>(a);
+}
+template <typename T, int K>
+static cudaError_t libmf_k(const LibmfLaunch& a) {
+  constexpr int S = (int)sizeof(T);
+  return launch_libmf_t<T, K, lanes_for(K, S, 16)>(a);
 }
 template <typename T, int K>
 static cudaError_t rmse_k(const RmseLaunch& a) {
@@ -394,6 +484,7 @@ static cudaError_t wavefront_k(const WavefrontLaunch& a) {
 cudaError_t launch_hogwild(const HogwildLaunch& a) { MF_DISPATCH(hogwild_k, a) }
 cudaError_t launch_wavefront(const WavefrontLaunch& a) { MF_DISPATCH(wavefront_k, a) }
 cudaError_t launch_rmse(const RmseLaunch& a) { MF_DISPATCH(rmse_k, a) }
+cudaError_t launch_libmf(const LibmfLaunch& a) { MF_DISPATCH(libmf_k, a) }
 int ring_window(int k, int storage) {
   const int S = storage == 0 ? 4 : 2;
   switch (k) {

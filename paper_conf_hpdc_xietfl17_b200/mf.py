@@ -16,7 +16,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(HERE, "libmf_b200.so")
 
 STORAGE = {"fp32": 0, "fp16": 1, "bf16": 2}
-SCHEDULE = {"hogwild": 0, "wavefront": 1}
+SCHEDULE = {"hogwild": 0, "wavefront": 1, "libmf": 2}
 SETS = {"train": 0, "test": 1}
 EXPORTS = {"perm": 0, "rho_r": 1, "rho_c": 2, "blockid": 3, "chunkorder": 4, "wfseq": 5,
            "tickets": 6, "strata": 7}
