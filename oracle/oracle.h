@@ -39,6 +39,12 @@ void   or_update(int32_t k, float* p, float* q, float r, float gamma,
                  float lambda_p, float lambda_q, int32_t storage); /* Alg. 1 l.8-10 */
 double or_sample_loss(int32_t k, const double* p, const double* q, double r,
                       double lambda_p, double lambda_q);           /* Eq. 3 */
+/* ADAGRAD variant ("cuMF_SGD can also use ADAGRAD", Duchi et al. [20]; reading R23):
+ * per coordinate, with pre-update values (R1):
+ *   g_p = -(e q - lambda_p p);  G_p += g_p^2;  p <- p - alpha g_p / sqrt(G_p + eps)   (same for q)
+ * gp, gq: the fp32 accumulators of p_u and q_v. */
+void   or_update_adagrad(int32_t k, float* p, float* q, float* gp, float* gq, float r,
+                         float alpha, float lambda_p, float lambda_q, float eps, int32_t storage);
 
 /* ---- a whole training run, in the schedule's serial order ---- */
 typedef struct or_params {
@@ -56,6 +62,8 @@ typedef struct or_params {
   int32_t wf_cols;         /* c: wavefront column sub-blocks per strata block */
   int32_t grid_a;          /* a: strata grid a x a (1 = single block) */
   int32_t cyclic;          /* wavefront cyclic column order variant (A: cyclic) */
+  int32_t lr_rule;         /* 0 = Eq. 9 schedule; 1 = ADAGRAD (or_update_adagrad, R23) */
+  float   ada_eps;         /* ADAGRAD epsilon */
 } or_params;
 
 typedef struct or_ctx or_ctx;

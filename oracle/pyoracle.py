@@ -42,7 +42,8 @@ class Params(ctypes.Structure):
                 ("seed", ctypes.c_uint64), ("schedule", ctypes.c_int32),
                 ("storage", ctypes.c_int32), ("workers", ctypes.c_int32),
                 ("batch_f", ctypes.c_int32), ("wf_cols", ctypes.c_int32),
-                ("grid_a", ctypes.c_int32), ("cyclic", ctypes.c_int32)]
+                ("grid_a", ctypes.c_int32), ("cyclic", ctypes.c_int32),
+                ("lr_rule", ctypes.c_int32), ("ada_eps", ctypes.c_float)]
 
 
 _lib = None
@@ -63,6 +64,7 @@ def lib() -> ctypes.CDLL:
             "or_bf16_bits": (ctypes.c_uint16, [f32]), "or_bf16_value": (f32, [ctypes.c_uint16]),
             "or_round_storage": (f32, [i32, f32]), "or_gamma": (f32, [f32, f32, i32]),
             "or_update": (None, [i32, vp, vp, f32, f32, f32, f32, i32]),
+            "or_update_adagrad": (None, [i32, vp, vp, vp, vp, f32, f32, f32, f32, f32, i32]),
             "or_sample_loss": (f64, [i32, vp, vp, f64, f64, f64]),
             "or_create": (vp, [ctypes.POINTER(Params), i64, vp, vp, vp]),
             "or_destroy": (None, [vp]), "or_train_epoch": (ctypes.c_int, [vp]),
@@ -99,6 +101,14 @@ def update(p, q, r, gamma, lambda_p, lambda_q, storage="fp32"):
     return p, q
 
 
+def update_adagrad(p, q, gp, gq, r, alpha, lambda_p, lambda_q, eps=1e-8, storage="fp32"):
+    """One ADAGRAD update (R23) on copies; returns (p', q', gp', gq')."""
+    p, q, gp, gq = (np.array(x, dtype=np.float32).copy() for x in (p, q, gp, gq))
+    lib().or_update_adagrad(len(p), _ptr(p), _ptr(q), _ptr(gp), _ptr(gq), r, alpha, lambda_p,
+                            lambda_q, eps, STORAGE[storage])
+    return p, q, gp, gq
+
+
 def sample_loss(p, q, r, lambda_p, lambda_q) -> float:
     p = np.ascontiguousarray(p, dtype=np.float64)
     q = np.ascontiguousarray(q, dtype=np.float64)
@@ -110,13 +120,15 @@ class Oracle:
 
     def __init__(self, m, n, k, u, v, r, *, lambda_p=0.05, lambda_q=None, alpha=0.08, beta=0.3,
                  init_scale=1.0, rating_scale=1.0, seed=42, schedule="hogwild", storage="fp32",
-                 workers=1, batch_f=256, wf_cols=0, grid_a=1, cyclic=False):
+                 workers=1, batch_f=256, wf_cols=0, grid_a=1, cyclic=False, lr_rule="eq9",
+                 ada_eps=1e-8):
         self.m, self.n, self.k = int(m), int(n), int(k)
         self.p = Params(m=m, n=n, k=k, lambda_p=lambda_p,
                         lambda_q=lambda_p if lambda_q is None else lambda_q, alpha=alpha,
                         beta=beta, init_scale=init_scale, rating_scale=rating_scale, seed=seed,
                         schedule=SCHEDULE[schedule], storage=STORAGE[storage], workers=workers,
-                        batch_f=batch_f, wf_cols=wf_cols, grid_a=grid_a, cyclic=int(cyclic))
+                        batch_f=batch_f, wf_cols=wf_cols, grid_a=grid_a, cyclic=int(cyclic),
+                        lr_rule={"eq9": 0, "adagrad": 1}[lr_rule], ada_eps=ada_eps)
         self.u = np.ascontiguousarray(u, dtype=np.int32)
         self.v = np.ascontiguousarray(v, dtype=np.int32)
         self.r = np.ascontiguousarray(r, dtype=np.float32)

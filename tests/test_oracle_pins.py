@@ -458,3 +458,60 @@ def test_create_rejects_bad_input():
         po.Oracle(10, 10, 4, [10], [0], [1.0])
     with pytest.raises(ValueError):
         po.Oracle(10, 10, 4, [0], [0], [float("nan")])
+
+
+# --------------------------------------------------------------------------- ADAGRAD (R23)
+
+def test_adagrad_first_step_is_alpha_sign():
+    """From zero accumulators each coordinate moves by exactly alpha against its gradient:
+    dp / sqrt(dp^2) = sign(dp).  Dyadic values: exact.  p=(1,2), q=(3,4), r=10, lambda=.5:
+    e = -1, dp = e q - l p = (-3.5, -5), dq = e p - l q = (-2.5, -4)."""
+    p, q, gp, gq = po.update_adagrad([1, 2], [3, 4], [0, 0], [0, 0], 10.0, 0.125, 0.5, 0.5, eps=0.0)
+    assert p.tolist() == [0.875, 1.875] and q.tolist() == [2.875, 3.875]
+    assert gp.tolist() == [12.25, 25.0] and gq.tolist() == [6.25, 16.0]
+
+
+def test_adagrad_reduces_to_plain_sgd_for_frozen_accumulators():
+    """With accumulators at 2^40 an fp32 G + g^2 (g^2 < 2^16) stays 2^40 and sqrt(G) = 2^20, so
+    the ADAGRAD step must equal Alg. 1's update with gamma = alpha * 2^-20 BIT-EXACTLY (scaling
+    by a power of two commutes with rounding)."""
+    rng = np.random.default_rng(8)
+    for _ in range(50):
+        k = int(rng.choice([1, 4, 16]))
+        p = rng.normal(size=k).astype(np.float32)
+        q = rng.normal(size=k).astype(np.float32)
+        r, a = float(rng.normal() * 3), float(np.float32(rng.uniform(0.01, 1)))
+        big = np.full(k, 2.0 ** 40, np.float32)
+        p1, q1, gp, gq = po.update_adagrad(p, q, big, big, r, a, 0.05, 0.07, eps=0.0)
+        p2, q2 = po.update(p, q, r, a * 2.0 ** -20, 0.05, 0.07)
+        assert np.array_equal(p1, p2) and np.array_equal(q1, q2)
+        assert np.array_equal(gp, big) and np.array_equal(gq, big)
+
+
+def test_adagrad_step_direction_is_the_eq3_gradient():
+    """(p' - p) sqrt(G') / alpha = -(1/2) grad_p of Eq. 3 (central differences, double)."""
+    rng = np.random.default_rng(9)
+    for _ in range(10):
+        k = 7
+        p = rng.normal(size=k).astype(np.float32)
+        q = rng.normal(size=k).astype(np.float32)
+        g0 = rng.uniform(0.5, 2.0, k).astype(np.float32)
+        r, a, lp, lq = 1.3, 0.01, 0.2, 0.3
+        p1, q1, gp, gq = po.update_adagrad(p, q, g0, g0, r, a, lp, lq, eps=0.0)
+        pd, qd, h = p.astype(np.float64), q.astype(np.float64), 1e-6
+        grad = np.array([(po.sample_loss(pd + h * e, qd, r, lp, lq) -
+                          po.sample_loss(pd - h * e, qd, r, lp, lq)) / (2 * h) for e in np.eye(k)])
+        step = (p1.astype(np.float64) - pd) * np.sqrt(gp.astype(np.float64)) / a
+        np.testing.assert_allclose(step, -0.5 * grad, rtol=3e-3, atol=3e-3)
+
+
+def test_adagrad_training_converges_on_tiny():
+    R = _tiny_set()
+    o = po.Oracle(R.m, R.n, 16, R.u, R.v, R.r, lambda_p=0.05, alpha=0.05, lr_rule="adagrad")
+    r0 = o.rmse(R.ut, R.vt, R.rt)
+    losses = [o.loss()]
+    for _ in range(10):
+        o.train_epoch()
+        losses.append(o.loss())
+    assert o.rmse(R.ut, R.vt, R.rt) < 0.5 * r0
+    assert losses[-1] < 0.2 * losses[0]
