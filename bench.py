@@ -48,6 +48,7 @@ def parse():
     ap.add_argument("--staged", action="store_true",
                     help="out-of-core: ratings in pinned host memory, streamed per stratum")
     ap.add_argument("--grid-a", type=int, default=0)
+    ap.add_argument("--lr-rule", default="eq9", choices=["eq9", "adagrad"])
     ap.add_argument("--batch-f", type=int, default=0,
                     help="Eq. 8 f (0 = 256 on 1 GPU, 1024 with strata; DESIGN.md section 7)")
     ap.add_argument("--fraction", type=float, default=1.0, help="scale the workload (testing)")
@@ -241,7 +242,8 @@ def main():
     kw = dict(schedule=args.schedule, storage=args.storage, workers=args.workers,
               wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes, prefetch=args.prefetch,
               wf_kernel=args.wf_kernel, staged=args.staged, grid_a=args.grid_a,
-              batch_f=args.batch_f or (1024 if world > 1 or args.grid_a > 1 else 256), seed=42,
+              batch_f=args.batch_f or (1024 if world > 1 or args.grid_a > 1 else 256),
+              lr_rule=args.lr_rule, seed=42,
               device=local, rank=rank, world=world, nccl_id=nccl_id, **hp)
     torch.cuda.synchronize()
     model = mf.MF(R.m, R.n, args.k, stream=stream, **kw)

@@ -93,6 +93,11 @@ typedef struct mf_params {
   int32_t cyclic;         /* wavefront: 1 = cyclic column order (A: cyclic variant), needs c >= s */
   int32_t lane_bytes;     /* Hogwild/RMSE kernel: bytes of p_u (and q_v) per lane, 16 or 32 (0 = 16) */
   int32_t prefetch;       /* Hogwild software-pipeline depth: samples in flight per worker, 1 or 2 (0 = 1) */
+  int32_t lr_rule;        /* 0 = Eq. 9 schedule (the paper); 1 = ADAGRAD (P:L419 future work,
+                             Duchi et al. [20]; R23): per-coordinate fp32 accumulators
+                             G += g^2, step alpha*g/sqrt(G + ada_eps); Hogwild and register
+                             wavefront kernels                                                  */
+  float ada_eps;          /* ADAGRAD epsilon (0 = 1e-8)                                         */
   int32_t staged;         /* 1 = out-of-core ratings (section 6.2): after the GPU
                              preprocessing the bucketed ratings live in pinned host memory and
                              each stratum's blocks stream into one of two HBM buffers on a copy

@@ -446,6 +446,8 @@ struct mf_ctx {
   // out-of-core staging (params.staged; section 6.2): the bucketed ratings live in
   // pinned host memory; each stratum's blocks are copied into one of two device buffers on a
   // copy stream while the previous stratum computes.
+  float* GP = nullptr;             // ADAGRAD accumulators (lr_rule 1), fp32, relabelled rows
+  float* GQ = nullptr;
   bool libmf = false;              // LIBMF-GPU table-scheduler baseline (MF_LIBMF)
   int64_t *d_blk_off = nullptr, *d_blk_len = nullptr;
   int *lm_lock = nullptr, *lm_row = nullptr, *lm_col = nullptr, *lm_done = nullptr, *lm_rem = nullptr;
@@ -663,6 +665,8 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->wf_kernel < 0 || p->wf_kernel > 2) return MF_E_INVAL;
   if (p->transport < 0 || p->transport > 1) return MF_E_INVAL;
   if (p->staged < 0 || p->staged > 1) return MF_E_INVAL;
+  if (p->lr_rule < 0 || p->lr_rule > 1 || !(p->ada_eps >= 0.f)) return MF_E_INVAL;
+  if (p->lr_rule == 1 && p->schedule == MF_LIBMF) return MF_E_UNSUPPORTED;
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
   const int a = p->grid_a > 0 ? p->grid_a : (libmf ? 64 : (world == 1 ? 1 : 8));
@@ -1135,6 +1139,12 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
     }
   }
   TRY(init_factors(c));
+  if (c->p.lr_rule == 1) {
+    TRY(c->alloc(&c->GP, (size_t)(c->m * c->k)));
+    TRY(c->alloc(&c->GQ, (size_t)(c->n * c->k)));
+    CUDA_TRY(c, cudaMemsetAsync(c->GP, 0, (size_t)(c->m * c->k) * 4, c->st));
+    CUDA_TRY(c, cudaMemsetAsync(c->GQ, 0, (size_t)(c->n * c->k) * 4, c->st));
+  }
   TRY(alloc_schedule(c));
   if (c->staged) TRY(setup_staging(c));
   CUDA_TRY(c, cudaStreamSynchronize(c->st));
@@ -1291,6 +1301,18 @@ static cudaEvent_t ev_at(mf_ctx* c, int i) {
 }
 
 // One strata block set (the blocks rank g trains in sub-epoch j) of epoch t.
+static AdaArgs ada_args(const mf_ctx* c) {
+  AdaArgs A{};
+  if (c->p.lr_rule == 1) {
+    A.GP = c->GP;
+    A.GQ = c->GQ;
+    A.lp = c->p.lambda_p;
+    A.lq = c->p.lambda_q;
+    A.eps = c->p.ada_eps > 0.f ? c->p.ada_eps : 1e-8f;
+  }
+  return A;
+}
+
 // shift of block b in the current staging buffer (0 when the ratings are resident)
 static int64_t slot_shift(const mf_ctx* c, int buf, int64_t b) {
   if (!c->staged) return 0;
@@ -1326,6 +1348,8 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     L.slots = slots; L.chunks = c->chunk_order; L.segs = segs; L.counter = c->counter;
     L.workers = c->p.workers; L.num_sms = c->num_sms; L.f = c->f;
     L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
+    L.ada = ada_args(c);
+    if (L.ada.GP) L.g = c->p.alpha;        // ADAGRAD: constant alpha, no Eq. 9 decay
     L.out_workers = &c->last_workers; L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
     CUDA_TRY(c, launch_hogwild(L));
@@ -1348,6 +1372,8 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     L.seq = c->seq + base; L.rank = c->rank_arr + base; L.tickets = c->tickets;
     L.s = c->s; L.c = c->c; L.num_sms = c->num_sms; L.P = c->P; L.Q = c->Q; L.g = g;
     L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
+    L.ada = ada_args(c);
+    if (L.ada.GP) L.g = c->p.alpha;
     L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
     cudaError_t e = launch_wavefront(L);
@@ -1521,7 +1547,7 @@ mf_status mf_get_stats(mf_ctx* c, mf_stats* out) {
   out->sgd_launches = c->n_sgd;
   out->launches = c->n_launch;
   out->updates = c->updates;
-  out->bytes_per_update = 12 + 4 * (int64_t)c->k * c->ssize();
+  out->bytes_per_update = 12 + 4 * (int64_t)c->k * c->ssize() + (c->GP ? 16 * (int64_t)c->k : 0);
   out->workers = c->last_workers;
   out->lanes = c->last_lanes;
   out->grid = c->last_grid;

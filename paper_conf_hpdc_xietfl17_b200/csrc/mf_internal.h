@@ -6,6 +6,7 @@
 #include <cstdint>
 
 #include "mf_common.cuh"
+#include "mf_sgd.cuh"
 
 namespace mfb {
 
@@ -29,6 +30,7 @@ struct HogwildLaunch {
   int workers, num_sms, f;
   void *P, *Q;
   float g, lp, lq;
+  AdaArgs ada;              // ada.GP != nullptr: ADAGRAD (g = alpha)
   cudaStream_t stream;
   int *out_workers, *out_lanes, *out_grid;
 };
@@ -47,6 +49,7 @@ struct WavefrontLaunch {
   int s, c, num_sms;
   void *P, *Q;
   float g, lp, lq;
+  AdaArgs ada;              // ada.GP != nullptr: ADAGRAD (register kernel; g = alpha)
   cudaStream_t stream;
   int *out_lanes, *out_grid;
 };

@@ -23,12 +23,12 @@ constexpr int ring_ahead(int K, int S) { return ring_slots(K, S) == 32 ? 15 : 7;
 // f consecutive slots of its chunk serially.  Persistent grid: workers loop until the list is
 // exhausted.  The chunk list of a launch is the concatenation of up to kMaxSegs block segments.
 // ---------------------------------------------------------------------------------------------
-template <typename T, int K, int L, int D>
+template <typename T, int K, int L, int D, bool ADA>
 __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slots,
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
                                                  unsigned long long* __restrict__ counter,
                                                  int workers, T* __restrict__ P, T* __restrict__ Q,
-                                                 int f, float g, float lp, float lq) {
+                                                 int f, float g, float lp, float lq, AdaArgs ada) {
   constexpr int GPW = 32 / L;
   const float cp = 1.f - g * lp, cq = 1.f - g * lq;
   const int lane = threadIdx.x & 31;
@@ -53,7 +53,8 @@ __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slot
       lo = (int64_t)chunk * f + segs.shift[sgi];
     }
     // every group of the warp runs f iterations in lockstep (inactive ones on sentinels)
-    run_serial<T, K, L, D, true>(slots, lo, f, act, P, Q, g, cp, cq, gl, gbase, 0xffffffffu);
+    run_serial<T, K, L, D, true, ADA>(slots, lo, f, act, P, Q, g, cp, cq, gl, gbase, 0xffffffffu,
+                                      ada);
   }
 }
 
@@ -94,14 +95,14 @@ __device__ __forceinline__ void ticket_release(int* t, int next, unsigned gmask,
   if (gl == 0) st_relaxed(t, next);
 }
 
-template <typename T, int K, int L>
+template <typename T, int K, int L, bool ADA>
 __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ slots,
                                                    const int64_t* __restrict__ sub_off,
                                                    const int32_t* __restrict__ seq,
                                                    const int32_t* __restrict__ rank,
                                                    int* __restrict__ tickets, int s, int c,
                                                    T* __restrict__ P, T* __restrict__ Q, float g,
-                                                   float lp, float lq, int64_t shift) {
+                                                   float lp, float lq, int64_t shift, AdaArgs ada) {
   const int lane = threadIdx.x & 31;
   const int grp = lane / L, gl = lane % L, gbase = grp * L;
   const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
@@ -116,8 +117,8 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
     ticket_acquire(tickets + col, tgt);
     const int64_t sb = (int64_t)worker * c + col;
     const int64_t lo = __ldg(sub_off + sb) + shift;
-    run_serial<T, K, L, 2, false>(slots, lo, (int)(__ldg(sub_off + sb + 1) + shift - lo), true, P, Q, g, cp,
-                                  cq, gl, gbase, gmask);
+    run_serial<T, K, L, 2, false, ADA>(slots, lo, (int)(__ldg(sub_off + sb + 1) + shift - lo), true, P,
+                                       Q, g, cp, cq, gl, gbase, gmask, ada);
     ticket_release(tickets + col, tgt + 1, gmask, gl);
   }
 }
@@ -305,9 +306,9 @@ __global__ void k_rmse_final(const double* __restrict__ partial, int n, double* 
 // ---------------------------------------------------------------------------------------------
 // Dispatch
 // ---------------------------------------------------------------------------------------------
-template <typename T, int K, int L, int D>
+template <typename T, int K, int L, int D, bool ADA = false>
 static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
-  auto kern = k_hogwild<T, K, L, D>;
+  auto kern = k_hogwild<T, K, L, D, ADA>;
   const int threads = 256;
   int per_sm = 0;
   cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, 0);
@@ -321,13 +322,13 @@ static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
   if (a.out_grid) *a.out_grid = blocks;
   kern<<<blocks, threads, 0, a.stream>>>(a.slots, a.chunks, a.segs, a.counter, workers,
                                          reinterpret_cast<T*>(a.P), reinterpret_cast<T*>(a.Q), a.f,
-                                         a.g, a.lp, a.lq);
+                                         a.g, a.lp, a.lq, a.ada);
   return cudaGetLastError();
 }
 
-template <typename T, int K, int L>
+template <typename T, int K, int L, bool ADA = false>
 static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
-  auto kern = k_wavefront<T, K, L>;
+  auto kern = k_wavefront<T, K, L, ADA>;
   const int threads = 128;
   const int64_t total_threads = (int64_t)a.s * L;
   const int blocks = (int)cdiv64(total_threads, threads);
@@ -347,7 +348,9 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
   T* Q = reinterpret_cast<T*>(a.Q);
   float g = a.g, lp = a.lp, lq = a.lq;
   int64_t shift = a.shift;
-  void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq, &shift};
+  AdaArgs ada = a.ada;
+  void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq, &shift,
+                  &ada};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, 0,
                                      a.stream);
 }
@@ -419,6 +422,7 @@ static constexpr int lanes_for(int K, int S, int LB) {
 template <typename T, int K, int LB>
 static cudaError_t hogwild_kl(const HogwildLaunch& a) {
   constexpr int S = (int)sizeof(T);
+  if (a.ada.GP) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, true>(a);
   if (a.prefetch == 1) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1>(a);
   return launch_hogwild_t<T, K, lanes_for(K, S, LB), 2>(a);
 }
@@ -440,6 +444,7 @@ static cudaError_t rmse_k(const RmseLaunch& a) {
 template <typename T, int K>
 static cudaError_t wavefront_k(const WavefrontLaunch& a) {
   constexpr int S = (int)sizeof(T);
+  if (a.ada.GP) return launch_wavefront_t<T, K, lanes_for(K, S, 8), true>(a);  // register kernel
   constexpr int L2 = ring_lanes(K, S);
   constexpr int L3 = L2 / 2;                 // lane_bytes = 32: half the lanes, 32 B per lane
   if constexpr (L3 > ring_ahead(K, S) && (K * S / L3) % 16 == 0)

@@ -48,6 +48,7 @@ class Params(ctypes.Structure):
                 ("batch_f", ctypes.c_int32), ("wf_cols", ctypes.c_int32),
                 ("grid_a", ctypes.c_int32), ("cyclic", ctypes.c_int32),
                 ("lane_bytes", ctypes.c_int32), ("prefetch", ctypes.c_int32),
+                ("lr_rule", ctypes.c_int32), ("ada_eps", ctypes.c_float),
                 ("staged", ctypes.c_int32), ("wf_kernel", ctypes.c_int32),
                 ("device", ctypes.c_int32),
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
@@ -183,6 +184,7 @@ class MF:
                  schedule: str = "hogwild", storage: str = "fp32", workers: int = 0,
                  batch_f: int = 256, wf_cols: int = 0, grid_a: int = 0, cyclic: bool = False,
                  lane_bytes: int = 0, prefetch: int = 0, wf_kernel: int = 0, staged: bool = False,
+                 lr_rule: str = "eq9", ada_eps: float = 1e-8,
                  device: int = 0, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, transport: int = 0, stream=None,
                  allocator: str = "torch"):
@@ -198,6 +200,7 @@ class MF:
         p.workers, p.batch_f, p.wf_cols, p.grid_a = workers, batch_f, wf_cols, grid_a
         p.cyclic, p.lane_bytes, p.prefetch, p.wf_kernel = int(cyclic), lane_bytes, prefetch, wf_kernel
         p.staged = int(staged)
+        p.lr_rule, p.ada_eps = {"eq9": 0, "adagrad": 1}[lr_rule], ada_eps
         p.device, p.rank, p.world, p.transport = device, rank, world, transport
         self._id_buf = None
         if nccl_id is not None:

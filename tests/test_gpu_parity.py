@@ -28,7 +28,7 @@ def pair(R, k=16, **kw):
     g.load(R.u, R.v, R.r, "train")
     if R.ut is not None:
         g.load(R.ut, R.vt, R.rt, "test")
-    okw = {kk: vv for kk, vv in kw.items() if kk not in ("lane_bytes", "prefetch", "wf_kernel")}
+    okw = {kk: vv for kk, vv in kw.items() if kk not in ("lane_bytes", "prefetch", "wf_kernel", "staged")}
     if kw.get("schedule") == "wavefront":
         okw.setdefault("workers", kw.get("workers"))
     o = po.Oracle(R.m, R.n, k, R.u, R.v, R.r, **okw)
@@ -345,3 +345,41 @@ def test_libmf_baseline_every_block_once_and_converges():
         assert g.stats()["updates"] == R.N
     rg, ro = g.rmse(), o.rmse(R.ut, R.vt, R.rt)
     assert abs(rg - ro) <= 0.01 * ro, (rg, ro)
+
+
+# ----------------------------------------------------------------------------- ADAGRAD (f4)
+
+@pytest.mark.parametrize("kw", [dict(schedule="wavefront", workers=8, wf_cols=16),
+                                dict(schedule="hogwild", workers=1),
+                                dict(schedule="wavefront", workers=4, wf_cols=5, grid_a=8)])
+def test_adagrad_deterministic_parity_fp32(tiny, kw):
+    """the same serial orders with the ADAGRAD step.  The step
+    alpha g / sqrt(G + eps) amplifies rounding differences of g by up to alpha/sqrt(eps) at the
+    first visit (G = 0), so the comparison uses eps = 1e-4 (amplification <= 5) and keeps the
+    north_star bars: |dP|,|dQ| <= 1e-4 after 1 epoch, RMSE relative <= 1e-5."""
+    common = dict(lambda_p=0.05, alpha=0.05, lr_rule="adagrad", ada_eps=1e-4)
+    g = mf.MF(tiny.m, tiny.n, 16, **common, **kw)
+    g.load(tiny.u, tiny.v, tiny.r)
+    g.load(tiny.ut, tiny.vt, tiny.rt, "test")
+    o = po.Oracle(tiny.m, tiny.n, 16, tiny.u, tiny.v, tiny.r, **common, **kw)
+    g.train_epoch()
+    o.train_epoch()
+    Pg, Qg = g.factors()
+    Po, Qo = o.factors()
+    assert np.abs(Pg - Po).max() <= 1e-4 and np.abs(Qg - Qo).max() <= 1e-4
+    rg, ro = g.rmse(), o.rmse(tiny.ut, tiny.vt, tiny.rt)
+    assert abs(rg - ro) <= 1e-5 * ro, (rg, ro)
+    assert g.stats()["bytes_per_update"] == 12 + 4 * 16 * 4 + 16 * 16
+
+
+def test_adagrad_hogwild_20_epochs_matches_oracle():
+    R = synth.powerlaw(4000, 900, 200_000, 20_000, seed=5, rank=8, mu=3.6, noise=0.5)
+    R = synth.Ratings(R.m, R.n, R.u.numpy(), R.v.numpy(), R.r.numpy(), R.ut.numpy(), R.vt.numpy(),
+                      R.rt.numpy())
+    common = dict(lambda_p=0.05, alpha=0.05, lr_rule="adagrad")
+    g, o = pair(R, k=32, schedule="hogwild", workers=32, **common)
+    for _ in range(20):
+        g.train_epoch()
+        o.train_epoch()
+    rg, ro = g.rmse(), o.rmse(R.ut, R.vt, R.rt)
+    assert abs(rg - ro) <= 0.005 * ro, (rg, ro)
