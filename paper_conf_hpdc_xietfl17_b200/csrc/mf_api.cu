@@ -660,7 +660,8 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (!(p->alpha >= 0.f) || !(p->beta >= 0.f) || !(p->lambda_p >= 0.f) || !(p->lambda_q >= 0.f))
     return MF_E_INVAL;
   if (!(p->rating_scale > 0.f) || !(p->init_scale > 0.f)) return MF_E_INVAL;
-  if (p->lane_bytes != 0 && p->lane_bytes != 16 && p->lane_bytes != 32) return MF_E_INVAL;
+  if (p->lane_bytes != 0 && p->lane_bytes != 16 && p->lane_bytes != 32 && p->lane_bytes != 64)
+    return MF_E_INVAL;
   if (p->prefetch < 0 || p->prefetch > 2) return MF_E_INVAL;
   if (p->wf_kernel < 0 || p->wf_kernel > 2) return MF_E_INVAL;
   if (p->transport < 0 || p->transport > 1) return MF_E_INVAL;
@@ -1134,7 +1135,7 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
     TRY(c->alloc(&c->dup, (size_t)std::max<int64_t>(c->nslots, 1)));
     if (N > 0) {
       k_dupdist<<<grid_for(N, c->num_sms), 256, 0, c->st>>>(c->slots, N, Gd,
-                                                          ring_window(c->k, c->p.storage), c->dup);
+                                                          ring_window(c->k, c->p.storage, c->p.lane_bytes), c->dup);
       KERNEL_TRY(c);
     }
   }

@@ -83,6 +83,6 @@ cudaError_t launch_hogwild(const HogwildLaunch& a);
 cudaError_t launch_libmf(const LibmfLaunch& a);
 cudaError_t launch_wavefront(const WavefrontLaunch& a);
 cudaError_t launch_rmse(const RmseLaunch& a);
-int ring_window(int k, int storage);  // history window W of k_wavefront2 for this geometry
+int ring_window(int k, int storage, int lane_bytes);  // history window W of k_wavefront2
 
 }  // namespace mfb

@@ -357,10 +357,10 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
 
 
 
-template <typename T, int K, int L>
+template <typename T, int K, int L, int RS_ = 0, int F_ = 0>
 static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
   constexpr int S = (int)sizeof(T);
-  constexpr int RS = ring_slots(K, S), F = ring_ahead(K, S);
+  constexpr int RS = RS_ ? RS_ : ring_slots(K, S), F = F_ ? F_ : ring_ahead(K, S);
   auto kern = k_wavefront2<T, K, L, RS, F>;
   constexpr int ROWB = K * S;
   const int threads = 32;                                    // one warp = one worker
@@ -414,6 +414,11 @@ static cudaError_t launch_rmse_t(const RmseLaunch& a) {
   return cudaGetLastError();
 }
 
+// the quarter-lane ring (lane_bytes = 64): L = ring_lanes / 4 lanes, RS = 16, F = 7 < L
+constexpr bool quarter_ring_ok(int K, int S) {
+  return ring_lanes(K, S) / 4 > 7 && (K * S / (ring_lanes(K, S) / 4)) % 16 == 0;
+}
+
 // lanes per sample for a given bytes-per-lane target: L = clamp(k*S/lane_bytes, 1, 32)
 static constexpr int lanes_for(int K, int S, int LB) {
   return (K * S / LB) >= 32 ? 32 : ((K * S / LB) < 1 ? 1 : (K * S / LB));
@@ -449,6 +454,9 @@ static cudaError_t wavefront_k(const WavefrontLaunch& a) {
   constexpr int L3 = L2 / 2;                 // lane_bytes = 32: half the lanes, 32 B per lane
   if constexpr (L3 > ring_ahead(K, S) && (K * S / L3) % 16 == 0)
     if (a.variant == 1 && a.dup && a.lane_bytes == 32) return launch_wavefront2_t<T, K, L3>(a);
+  constexpr int L4 = L2 / 4;                 // lane_bytes = 64: a quarter of the lanes
+  if constexpr (quarter_ring_ok(K, S))
+    if (a.variant == 1 && a.dup && a.lane_bytes == 64) return launch_wavefront2_t<T, K, L4, 16, 7>(a);
   if constexpr (L2 > ring_ahead(K, S) && (K * S / L2) % 16 == 0)  // needs F < L, 16-B pieces
     if (a.variant == 1 && a.dup) return launch_wavefront2_t<T, K, L2>(a);
   return launch_wavefront_t<T, K, lanes_for(K, S, 8)>(a);
@@ -490,14 +498,20 @@ cudaError_t launch_hogwild(const HogwildLaunch& a) { MF_DISPATCH(hogwild_k, a) }
 cudaError_t launch_wavefront(const WavefrontLaunch& a) { MF_DISPATCH(wavefront_k, a) }
 cudaError_t launch_rmse(const RmseLaunch& a) { MF_DISPATCH(rmse_k, a) }
 cudaError_t launch_libmf(const LibmfLaunch& a) { MF_DISPATCH(libmf_k, a) }
-int ring_window(int k, int storage) {
-  const int S = storage == 0 ? 4 : 2;
+template <int K, int S>
+static int ring_window_t(int lane_bytes) {
+  if (lane_bytes == 64 && quarter_ring_ok(K, S)) return 16 - 7 - 1;  // RS = 16, F = 7
+  return ring_slots(K, S) - ring_ahead(K, S) - 1;
+}
+
+int ring_window(int k, int storage, int lane_bytes) {
+  const bool h = storage != 0;
   switch (k) {
-    case 16: return ring_slots(16, S) - ring_ahead(16, S) - 1;
-    case 32: return ring_slots(32, S) - ring_ahead(32, S) - 1;
-    case 64: return ring_slots(64, S) - ring_ahead(64, S) - 1;
-    case 128: return ring_slots(128, S) - ring_ahead(128, S) - 1;
-    default: return ring_slots(256, S) - ring_ahead(256, S) - 1;
+    case 16: return h ? ring_window_t<16, 2>(lane_bytes) : ring_window_t<16, 4>(lane_bytes);
+    case 32: return h ? ring_window_t<32, 2>(lane_bytes) : ring_window_t<32, 4>(lane_bytes);
+    case 64: return h ? ring_window_t<64, 2>(lane_bytes) : ring_window_t<64, 4>(lane_bytes);
+    case 128: return h ? ring_window_t<128, 2>(lane_bytes) : ring_window_t<128, 4>(lane_bytes);
+    default: return h ? ring_window_t<256, 2>(lane_bytes) : ring_window_t<256, 4>(lane_bytes);
   }
 }
 

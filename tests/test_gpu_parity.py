@@ -106,10 +106,13 @@ def test_deterministic_one_epoch_parity_fp32(tiny, kw):
     assert abs(rg - ro) <= 1e-5 * ro
 
 
-@pytest.mark.parametrize("k,wfk", [(32, 0), (64, 0), (128, 0), (256, 0), (128, 2)])
-def test_deterministic_parity_other_k_ragged(k, wfk):
+@pytest.mark.parametrize("k,wfk,lb", [(32, 0, 0), (64, 0, 0), (128, 0, 0), (256, 0, 0), (128, 2, 0),
+                                      (128, 0, 32), (128, 0, 64), (256, 0, 64)])
+def test_deterministic_parity_other_k_ragged(k, wfk, lb):
+    """lb: ring geometry (0 = 32 lanes x 16 B, 32 = half the lanes, 64 = a quarter, RS 16)."""
     R = ragged()
-    g, o = pair(R, k=k, schedule="wavefront", workers=6, wf_cols=9, wf_kernel=wfk, **TABLE3_NETFLIX)
+    g, o = pair(R, k=k, schedule="wavefront", workers=6, wf_cols=9, wf_kernel=wfk, lane_bytes=lb,
+                **TABLE3_NETFLIX)
     for _ in range(2):
         g.train_epoch()
         o.train_epoch()
