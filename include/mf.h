@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define MF_ABI_VERSION 1
+#define MF_ABI_VERSION 2
 
 typedef struct mf_ctx mf_ctx; /* opaque, owned by the library */
 
@@ -114,6 +114,12 @@ typedef struct mf_params {
                              for loopback any key naming the group                              */
   void* stream;           /* cudaStream_t or NULL                                               */
   const mf_allocator* alloc; /* NULL = cudaMallocAsync                                          */
+  int32_t launch_blocks;  /* Hogwild: strata blocks per SGD launch (0 = every block the rank
+                             trains in the sub-epoch, interleaved in one launch).  B > 0 runs
+                             them B at a time, in row-segment order: with world = 1 and B = a/G
+                             each launch is exactly what one of G GPUs runs in that sub-epoch
+                             (tools/scale_emulation.py).  Same result either way: a stratum's
+                             blocks touch disjoint P and Q rows                                 */
 } mf_params;
 
 /* Fill *p with defaults (Table 3 Netflix lambda/alpha/beta, k = 128, fp32, Hogwild, f = 256). */
@@ -186,6 +192,11 @@ typedef struct mf_stats {
   int32_t workers, lanes, grid, block;
 } mf_stats;
 mf_status mf_get_stats(mf_ctx* ctx, mf_stats* out);
+
+/* Per-launch device times (ms, CUDA events) of the SGD launches of the last epoch, in launch
+ * order (synchronises).  With ms == NULL only *n is set; otherwise *n must be >= the count and
+ * receives it. */
+mf_status mf_get_launch_ms(mf_ctx* ctx, double* ms, int64_t* n);
 
 /* Host-only strata planner (no GPU needed): which rank trains block row-segment r in
  * sub-epoch j of epoch t, and which Q segments move before sub-epoch j.  For each segment

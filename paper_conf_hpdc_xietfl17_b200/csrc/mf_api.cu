@@ -663,7 +663,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->lane_bytes != 0 && p->lane_bytes != 16 && p->lane_bytes != 32 && p->lane_bytes != 64)
     return MF_E_INVAL;
   if (p->prefetch < 0 || p->prefetch > 2) return MF_E_INVAL;
-  if (p->wf_kernel < 0 || p->wf_kernel > 2) return MF_E_INVAL;
+  if (p->wf_kernel < 0 || p->wf_kernel > 2 || p->launch_blocks < 0) return MF_E_INVAL;
   if (p->transport < 0 || p->transport > 1) return MF_E_INVAL;
   if (p->staged < 0 || p->staged > 1) return MF_E_INVAL;
   if (p->lr_rule < 0 || p->lr_rule > 1 || !(p->ada_eps >= 0.f)) return MF_E_INVAL;
@@ -1322,6 +1322,33 @@ static int64_t slot_shift(const mf_ctx* c, int buf, int64_t b) {
   return 0;
 }
 
+// Level table of the interleaved claim order (ChunkSegs): level l runs, round-robin over the
+// segments whose length exceeds the previous level's, the chunk indices up to the next
+// distinct segment length.
+static void finalize_segs(ChunkSegs& s) {
+  std::vector<int64_t> lens;
+  for (int i = 0; i < s.n; ++i) lens.push_back(s.prefix[i + 1] - s.prefix[i]);
+  std::vector<int64_t> cuts(lens);
+  std::sort(cuts.begin(), cuts.end());
+  cuts.erase(std::unique(cuts.begin(), cuts.end()), cuts.end());
+  s.nlev = 0;
+  int64_t lo = 0, base = 0;
+  for (int64_t cut : cuts) {
+    const int l = s.nlev;
+    int cnt = 0;
+    for (int i = 0; i < s.n; ++i)
+      if (lens[(size_t)i] >= cut) s.lev_seg[l][cnt++] = (int8_t)i;
+    s.lev_base[l] = base;
+    s.lev_lo[l] = lo;
+    s.lev_cnt[l] = cnt;
+    base += (cut - lo) * cnt;
+    lo = cut;
+    ++s.nlev;
+  }
+  s.lev_base[s.nlev] = base;                 // == prefix[n]
+  for (int l = s.nlev + 1; l <= kMaxSegs; ++l) s.lev_base[l] = base;
+}
+
 static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, float g, int buf) {
   const Rating* slots = c->staged ? c->stg[buf] : c->slots;
   const uint16_t* dup = c->staged ? c->stg_dup[buf] : c->dup;
@@ -1339,9 +1366,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
       ++segs.n;
     }
     if (segs.n == 0) return MF_OK;
-    segs.minlen = segs.prefix[1] - segs.prefix[0];
-    for (int s2 = 1; s2 < segs.n; ++s2)
-      segs.minlen = std::min(segs.minlen, segs.prefix[s2 + 1] - segs.prefix[s2]);
+    finalize_segs(segs);
     CUDA_TRY(c, cudaMemsetAsync(c->counter, 0, sizeof(unsigned long long), c->st));
     HogwildLaunch L{};
     L.storage = c->p.storage; L.k = c->k; L.lane_bytes = c->p.lane_bytes ? c->p.lane_bytes : 16;
@@ -1514,7 +1539,11 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
       TRY(stage(c, last ? t + 1 : t, last ? 0 : j + 1, 1 - buf));   // overlap the next copy
       CUDA_TRY(c, cudaStreamWaitEvent(c->st, c->ev_h2d[buf], 0));
     }
-    TRY(run_stratum(c, std::vector<int64_t>(blocks.begin(), blocks.begin() + nb), g, buf));
+    const int per_launch = (!c->wf && c->p.launch_blocks > 0) ? c->p.launch_blocks : std::max(nb, 1);
+    for (int b0 = 0; b0 < nb; b0 += per_launch)
+      TRY(run_stratum(c, std::vector<int64_t>(blocks.begin() + b0,
+                                              blocks.begin() + std::min(nb, b0 + per_launch)),
+                      g, buf));
     if (c->staged) {
       CUDA_TRY(c, cudaEventRecord(c->ev_free[buf], c->st));
       c->cur_buf = 1 - buf;
@@ -1524,6 +1553,26 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   c->t = t + 1;
   c->have_stats = true;
   if (epoch_done) *epoch_done = c->t;
+  return MF_OK;
+}
+
+mf_status mf_get_launch_ms(mf_ctx* c, double* ms, int64_t* n) {
+  if (!c || !n) return MF_E_INVAL;
+  TRY(c->enter());
+  const int64_t cnt = c->have_stats ? c->n_sgd : 0;
+  if (!ms) {
+    *n = cnt;
+    return MF_OK;
+  }
+  if (*n < cnt) return MF_E_INVAL;
+  *n = cnt;
+  if (cnt == 0) return MF_OK;
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  for (int64_t i = 0; i < cnt; ++i) {
+    float x = 0.f;
+    CUDA_TRY(c, cudaEventElapsedTime(&x, c->ev[(size_t)(2 * i)], c->ev[(size_t)(2 * i + 1)]));
+    ms[i] = x;
+  }
   return MF_OK;
 }
 

@@ -17,8 +17,17 @@ struct ChunkSegs {
   int64_t begin[kMaxSegs];
   int64_t prefix[kMaxSegs + 1];
   int64_t shift[kMaxSegs];  // slot of chunk q = q*f + shift (0 resident; staged: buffer offset)
-  int64_t minlen;           // shortest segment (chunks): claims interleave the segments
   int n;
+  // Claim order interleaves the segments (a stratum's blocks touch disjoint P and Q rows, so
+  // any interleaving gives the same result as running them one after another): level l covers
+  // claim positions [lev_base[l], lev_base[l+1]) and chunk indices [lev_lo[l], ...) of the
+  // lev_cnt[l] segments lev_seg[l][0..cnt) that are still that long, round-robin.  Built by
+  // finalize_segs() (mf_api.cu).
+  int nlev;
+  int64_t lev_base[kMaxSegs + 1];
+  int64_t lev_lo[kMaxSegs];
+  int32_t lev_cnt[kMaxSegs];
+  int8_t lev_seg[kMaxSegs][kMaxSegs];
 };
 
 struct HogwildLaunch {

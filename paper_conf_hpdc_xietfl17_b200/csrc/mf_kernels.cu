@@ -46,10 +46,13 @@ __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slot
     const int64_t ci = (int64_t)base + grp;
     const bool act = grp < nact && ci < total;
     int64_t lo = 0;
-    if (act) {
-      int sgi = 0;
-      while (ci >= segs.prefix[sgi + 1]) ++sgi;
-      const uint32_t chunk = __ldg(chunks + segs.begin[sgi] + (ci - segs.prefix[sgi]));
+    if (act) {                                       // claim position -> (block, chunk)
+      int lv = 0;
+      while (ci >= segs.lev_base[lv + 1]) ++lv;
+      const int64_t pos = ci - segs.lev_base[lv];
+      const int cnt = segs.lev_cnt[lv];
+      const int sgi = segs.lev_seg[lv][(int)(pos % cnt)];
+      const uint32_t chunk = __ldg(chunks + segs.begin[sgi] + segs.lev_lo[lv] + pos / cnt);
       lo = (int64_t)chunk * f + segs.shift[sgi];
     }
     // every group of the warp runs f iterations in lockstep (inactive ones on sentinels)

@@ -53,7 +53,8 @@ class Params(ctypes.Structure):
                 ("device", ctypes.c_int32),
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("transport", ctypes.c_int32), ("nccl_id", ctypes.c_void_p),
-                ("stream", ctypes.c_void_p), ("alloc", ctypes.POINTER(Allocator))]
+                ("stream", ctypes.c_void_p), ("alloc", ctypes.POINTER(Allocator)),
+                ("launch_blocks", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -68,7 +69,7 @@ class Stats(ctypes.Structure):
 _lib = None
 EXPORTED = ["mf_abi_version", "mf_params_default", "mf_create", "mf_load_coo", "mf_train_epoch",
             "mf_rmse", "mf_get_factors", "mf_set_factors", "mf_set_epoch", "mf_get_epoch",
-            "mf_export_schedule", "mf_get_stats", "mf_strata_holders", "mf_strata_plan",
+            "mf_export_schedule", "mf_get_stats", "mf_get_launch_ms", "mf_strata_holders", "mf_strata_plan",
             "mf_destroy",
             "mf_last_error", "mf_status_string"]
 
@@ -96,6 +97,7 @@ def lib() -> ctypes.CDLL:
         "mf_get_epoch": (i32, [vp, ctypes.POINTER(i32)]),
         "mf_export_schedule": (i32, [vp, i32, i32, vp, ctypes.POINTER(i64)]),
         "mf_get_stats": (i32, [vp, ctypes.POINTER(Stats)]),
+        "mf_get_launch_ms": (i32, [vp, vp, ctypes.POINTER(i64)]),
         "mf_strata_holders": (i32, [u64, i32, i32, i32, i32, vp]),
         "mf_strata_plan": (i32, [u64, i32, i32, i32, i64, i32, i32, vp, vp, vp, vp, vp]),
         "mf_destroy": (None, [vp]),
@@ -184,7 +186,7 @@ class MF:
                  schedule: str = "hogwild", storage: str = "fp32", workers: int = 0,
                  batch_f: int = 256, wf_cols: int = 0, grid_a: int = 0, cyclic: bool = False,
                  lane_bytes: int = 0, prefetch: int = 0, wf_kernel: int = 0, staged: bool = False,
-                 lr_rule: str = "eq9", ada_eps: float = 1e-8,
+                 lr_rule: str = "eq9", ada_eps: float = 1e-8, launch_blocks: int = 0,
                  device: int = 0, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, transport: int = 0, stream=None,
                  allocator: str = "torch"):
@@ -200,6 +202,7 @@ class MF:
         p.workers, p.batch_f, p.wf_cols, p.grid_a = workers, batch_f, wf_cols, grid_a
         p.cyclic, p.lane_bytes, p.prefetch, p.wf_kernel = int(cyclic), lane_bytes, prefetch, wf_kernel
         p.staged = int(staged)
+        p.launch_blocks = launch_blocks
         p.lr_rule, p.ada_eps = {"eq9": 0, "adagrad": 1}[lr_rule], ada_eps
         p.device, p.rank, p.world, p.transport = device, rank, world, transport
         self._id_buf = None
@@ -303,6 +306,15 @@ class MF:
         buf = np.empty(max(n.value, 1), dtype=np.int64)
         self._check(lib().mf_export_schedule(self.h, EXPORTS[what], epoch, buf.ctypes.data,
                                              ctypes.byref(n)), f"export({what})")
+        return buf[:n.value]
+
+    def launch_ms(self) -> np.ndarray:
+        """Device time (ms) of each SGD launch of the last epoch, in launch order."""
+        n = ctypes.c_int64(0)
+        self._check(lib().mf_get_launch_ms(self.h, None, ctypes.byref(n)), "mf_get_launch_ms")
+        buf = np.zeros(max(n.value, 1), dtype=np.float64)
+        self._check(lib().mf_get_launch_ms(self.h, buf.ctypes.data, ctypes.byref(n)),
+                    "mf_get_launch_ms")
         return buf[:n.value]
 
     def stats(self) -> dict:

@@ -28,7 +28,8 @@ def pair(R, k=16, **kw):
     g.load(R.u, R.v, R.r, "train")
     if R.ut is not None:
         g.load(R.ut, R.vt, R.rt, "test")
-    okw = {kk: vv for kk, vv in kw.items() if kk not in ("lane_bytes", "prefetch", "wf_kernel", "staged")}
+    okw = {kk: vv for kk, vv in kw.items() if kk not in ("lane_bytes", "prefetch", "wf_kernel", "staged",
+                                                          "launch_blocks")}
     if kw.get("schedule") == "wavefront":
         okw.setdefault("workers", kw.get("workers"))
     o = po.Oracle(R.m, R.n, k, R.u, R.v, R.r, **okw)
@@ -88,6 +89,8 @@ DET_CASES = [
     dict(schedule="wavefront", workers=4, wf_cols=5, grid_a=8),
     dict(schedule="hogwild", workers=1),
     dict(schedule="hogwild", workers=1, grid_a=8, batch_f=64),
+    dict(schedule="hogwild", workers=1, grid_a=8, batch_f=64, launch_blocks=3),
+    dict(schedule="hogwild", workers=1, grid_a=4, batch_f=16),
     dict(schedule="hogwild", workers=1, lane_bytes=32),
     dict(schedule="hogwild", workers=1, prefetch=2),
 ]
