@@ -48,6 +48,8 @@ def parse():
     ap.add_argument("--staged", action="store_true",
                     help="out-of-core: ratings in pinned host memory, streamed per stratum")
     ap.add_argument("--grid-a", type=int, default=0)
+    ap.add_argument("--q-atomic", type=int, default=0,
+                    help="Hogwild q_v write: 0 = plain store (paper), 1 = atomic delta (Hogwild! [44])")
     ap.add_argument("--lr-rule", default="eq9", choices=["eq9", "adagrad"])
     ap.add_argument("--batch-f", type=int, default=0,
                     help="Eq. 8 f (0 = 256 on 1 GPU, 1024 with strata; DESIGN.md section 7)")
@@ -217,7 +219,7 @@ def config_of(args, R):
             "storage": args.storage, "schedule": args.schedule,
             "batch_f": args.batch_f or (1024 if args.gpus > 1 or args.grid_a > 1 else 256),
             "parallelism": f"dsgd-strata{args.gpus}" if args.gpus > 1 else "1gpu",
-            "staged": bool(args.staged), "grid_a": args.grid_a or (8 if args.gpus > 1 else 1),
+            "staged": bool(args.staged), "q_atomic": bool(args.q_atomic), "grid_a": args.grid_a or (8 if args.gpus > 1 else 1),
             "l2": "inputs larger than L2 (COO %.2f GB per epoch); model P+Q stays cached as in "
                   "any training run" % (R.N * 12 / 1e9)}
 
@@ -243,7 +245,7 @@ def main():
               wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes, prefetch=args.prefetch,
               wf_kernel=args.wf_kernel, staged=args.staged, grid_a=args.grid_a,
               batch_f=args.batch_f or (1024 if world > 1 or args.grid_a > 1 else 256),
-              lr_rule=args.lr_rule, seed=42,
+              lr_rule=args.lr_rule, seed=42, q_atomic=bool(args.q_atomic),
               device=local, rank=rank, world=world, nccl_id=nccl_id, **hp)
     torch.cuda.synchronize()
     model = mf.MF(R.m, R.n, args.k, stream=stream, **kw)

@@ -29,8 +29,12 @@ ap.add_argument("--workload", default="netflix")
 ap.add_argument("--fraction", type=float, default=1.0)
 ap.add_argument("--epochs", type=int, default=3)
 ap.add_argument("--storage", default="fp16")
-ap.add_argument("--batch-f", type=int, default=1024)
+ap.add_argument("--batch-f", type=int, default=256)
 ap.add_argument("--out", default=None)
+ap.add_argument("--gs", default="1,2,4,8", help="GPU counts to emulate")
+ap.add_argument("--workers", default="0", help="comma list of Hogwild worker counts (0 = all resident)")
+ap.add_argument("--no-base", action="store_true")
+ap.add_argument("--q-atomic", action="store_true")
 args = ap.parse_args()
 
 s = synth.SHAPES[args.workload]
@@ -43,7 +47,7 @@ t_comm = 20e-3 + msg / 770e9 * 1e3          # ms per sub-epoch
 
 
 def run(**kw):
-    g = mf.MF(R.m, R.n, K, storage=args.storage, seed=42, **hp, **kw)
+    g = mf.MF(R.m, R.n, K, storage=args.storage, seed=42, q_atomic=args.q_atomic, **hp, **kw)
     g.load(R.u, R.v, R.r)
     g.load(R.ut, R.vt, R.rt, "test")
     g.train_epoch()                          # warm-up
@@ -54,22 +58,26 @@ def run(**kw):
     rmse = g.rmse()
     upd = g.stats()["updates"]
     g.close()
+    del g
+    torch.cuda.empty_cache()                 # the next ctx needs the 37 GB slot array again
     return np.array(per), rmse, upd
 
 
 rows = []
-base, rmse1, upd = run(grid_a=1, batch_f=256)
-t1 = float(base.sum(1).mean())
-rows.append(dict(G=1, grid="a=1 f=256", ms_epoch=t1, gups=upd / t1 / 1e6, rmse=rmse1))
-print(json.dumps(rows[-1]), flush=True)
-for G in (1, 2, 4, 8):
-    per, rmse, upd = run(grid_a=A, batch_f=args.batch_f, launch_blocks=A // G)
+t1 = float("nan")
+if not args.no_base:
+    base, rmse1, upd = run(grid_a=1, batch_f=256)
+    t1 = float(base.sum(1).mean())
+    rows.append(dict(G=1, grid="a=1 f=256", ms_epoch=t1, gups=upd / t1 / 1e6, rmse=rmse1))
+    print(json.dumps(rows[-1]), flush=True)
+for G, W in [(int(g), int(w)) for g in args.gs.split(",") for w in args.workers.split(",")]:
+    per, rmse, upd = run(grid_a=A, batch_f=args.batch_f, launch_blocks=A // G, workers=W)
     assert per.shape[1] == A * G, per.shape
     t = per.reshape(per.shape[0], A, G)                     # [epoch, sub-epoch j, rank g]
     comp = float(t.max(2).sum(1).mean())
     imb = float((t.max(2) / t.mean(2)).mean())
     tg = comp + (A * t_comm if G > 1 else 0.0)
-    rows.append(dict(G=G, grid=f"a={A} f={args.batch_f} blocks/launch={A // G}",
+    rows.append(dict(G=G, workers=W, grid=f"a={A} f={args.batch_f} blocks/launch={A // G}",
                      compute_ms=comp, comm_ms_est=A * t_comm if G > 1 else 0.0, ms_epoch=tg,
                      gups=upd / tg / 1e6, per_gpu_gups=upd / tg / 1e6 / G,
                      efficiency_vs_a1=(upd / tg) / (G * upd / t1), load_imbalance=imb, rmse=rmse))
