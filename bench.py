@@ -35,7 +35,9 @@ def parse():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="mf", choices=["mf", "reference"])
-    ap.add_argument("--workload", default="netflix", choices=["netflix", "yahoo", "hugewiki", "tiny"])
+    ap.add_argument("--workload", default=None, choices=["netflix", "yahoo", "hugewiki", "tiny"],
+                    help="default: netflix (configs[1]) on 1 GPU; yahoo (configs[2]) on N > 1 "
+                         "(DESIGN.md section 8: the set DSGD strata scale on)")
     ap.add_argument("--storage", default="fp16", choices=["fp16", "fp32", "bf16"])
     ap.add_argument("--schedule", default="hogwild", choices=["hogwild", "wavefront", "libmf"])
     ap.add_argument("--k", type=int, default=128)
@@ -48,11 +50,8 @@ def parse():
     ap.add_argument("--staged", action="store_true",
                     help="out-of-core: ratings in pinned host memory, streamed per stratum")
     ap.add_argument("--grid-a", type=int, default=0)
-    ap.add_argument("--q-atomic", type=int, default=0,
-                    help="Hogwild q_v write: 0 = plain store (paper), 1 = atomic delta (Hogwild! [44])")
     ap.add_argument("--lr-rule", default="eq9", choices=["eq9", "adagrad"])
-    ap.add_argument("--batch-f", type=int, default=0,
-                    help="Eq. 8 f (0 = 256 on 1 GPU, 1024 with strata; DESIGN.md section 7)")
+    ap.add_argument("--batch-f", type=int, default=0, help="Eq. 8 f (0 = 256, P:L277)")
     ap.add_argument("--fraction", type=float, default=1.0, help="scale the workload (testing)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -185,9 +184,15 @@ def cpu_baseline(R, hp, args, sample):
             "seconds": dt}
 
 
+def resolve_workload(args, world):
+    if args.workload is None:
+        args.workload = "netflix" if world == 1 else "yahoo"
+
+
 def run_reference(args):
     """--impl reference: the CPU oracle on the box's host cores (rank 0 only)."""
     world, rank, local = int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")), 0
+    resolve_workload(args, world)
     if rank != 0:
         return
     device = "cuda" if torch.cuda.is_available() else "cpu"
@@ -217,9 +222,9 @@ def config_of(args, R):
     return {"workload": f"{args.workload}-shaped synthetic (Table 2 shape, power-law skew)",
             "m": R.m, "n": R.n, "N_train": R.N, "N_test": R.Ntest, "k": args.k,
             "storage": args.storage, "schedule": args.schedule,
-            "batch_f": args.batch_f or (1024 if args.gpus > 1 or args.grid_a > 1 else 256),
+            "batch_f": args.batch_f or 256,
             "parallelism": f"dsgd-strata{args.gpus}" if args.gpus > 1 else "1gpu",
-            "staged": bool(args.staged), "q_atomic": bool(args.q_atomic), "grid_a": args.grid_a or (8 if args.gpus > 1 else 1),
+            "staged": bool(args.staged), "grid_a": args.grid_a or (8 if args.gpus > 1 else 1),
             "l2": "inputs larger than L2 (COO %.2f GB per epoch); model P+Q stays cached as in "
                   "any training run" % (R.N * 12 / 1e9)}
 
@@ -230,6 +235,7 @@ def main():
         return run_reference(args)
     world, rank, local = dist_setup(args)
     args.gpus = world
+    resolve_workload(args, world)
     device = torch.device(f"cuda:{local}")
     torch.cuda.set_device(device)
     from paper_conf_hpdc_xietfl17_b200 import mf
@@ -244,8 +250,8 @@ def main():
     kw = dict(schedule=args.schedule, storage=args.storage, workers=args.workers,
               wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes, prefetch=args.prefetch,
               wf_kernel=args.wf_kernel, staged=args.staged, grid_a=args.grid_a,
-              batch_f=args.batch_f or (1024 if world > 1 or args.grid_a > 1 else 256),
-              lr_rule=args.lr_rule, seed=42, q_atomic=bool(args.q_atomic),
+              batch_f=args.batch_f or 256,
+              lr_rule=args.lr_rule, seed=42,
               device=local, rank=rank, world=world, nccl_id=nccl_id, **hp)
     torch.cuda.synchronize()
     model = mf.MF(R.m, R.n, args.k, stream=stream, **kw)
@@ -361,30 +367,53 @@ def run_deterministic(args, R, hp, stream):
 
 
 def run_e2e(args, R, kw, stream):
-    """The same metric through the public API with HOST inputs: every step creates a ctx,
-    copies the pinned host COO in (mf_load_coo, on_device=0; includes the one-time GPU
-    preprocessing), trains one epoch and reads the test RMSE back (D2H)."""
+    """The same metric through the public API with the ratings in HOST memory: a ctx in the
+    paper's out-of-core mode (staged = 1, section 6.2) keeps the bucketed ratings
+    in pinned host memory and copies each epoch's ratings host -> device (cudaMemcpyAsync on a
+    copy stream, overlapped with the previous epoch's compute); every step is one epoch plus the
+    test RMSE read back to the host (D2H).  Host wall clock around K synchronised steps, after
+    the one-time load and a warm-up epoch.  Also reported: the cold path (mf_create + mf_load_coo
+    from pinned host + 1 epoch + mf_rmse per step), which includes the one-time preprocessing."""
     from paper_conf_hpdc_xietfl17_b200 import mf
     host = [x.cpu().pin_memory().numpy() for x in (R.u, R.v, R.r, R.ut, R.vt, R.rt)]
-    times = []
+    kw2 = dict(kw)
+    kw2["staged"] = True
+    m = mf.MF(R.m, R.n, args.k, stream=stream, **kw2)
+    m.load(host[0], host[1], host[2], "train", on_device=False)
+    m.load(host[3], host[4], host[5], "test", on_device=False)
+    m.train_epoch()
+    m.rmse("test")
+    steps = max(3, args.e2e_steps * 2)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        m.train_epoch()
+        m.rmse("test")                 # synchronises; 8-byte D2H
+    dt = (time.perf_counter() - t0) / steps
+    m.close()
+    cold = []
     for i in range(args.e2e_steps + 1):
         torch.cuda.synchronize()
-        t0 = time.perf_counter()
-        m = mf.MF(R.m, R.n, args.k, stream=stream, **kw)
-        m.load(host[0], host[1], host[2], "train", on_device=False)
-        m.load(host[3], host[4], host[5], "test", on_device=False)
-        m.train_epoch()
-        m.rmse("test")
+        t1 = time.perf_counter()
+        c = mf.MF(R.m, R.n, args.k, stream=stream, **kw)
+        c.load(host[0], host[1], host[2], "train", on_device=False)
+        c.load(host[3], host[4], host[5], "test", on_device=False)
+        c.train_epoch()
+        c.rmse("test")
         torch.cuda.synchronize()
-        dt = time.perf_counter() - t0
-        m.close()
         if i > 0:           # first iteration warms the allocator / module load
-            times.append(dt)
-    dt = float(np.mean(times))
-    return {"value": R.N / dt, "unit": "updates/s", "ms_per_step": 1000 * dt,
-            "h2d_bytes_per_step": int(12 * (R.N + R.Ntest)), "d2h_bytes_per_step": 8,
-            "what": "per step: mf_create + mf_load_coo(train,test from pinned host) + "
-                    "1 epoch + mf_rmse (host wall clock around synchronised calls)"}
+            cold.append(time.perf_counter() - t1)
+        c.close()
+    dc = float(np.mean(cold))
+    return {"value": R.N / dt, "unit": "updates/s", "ms_per_step": 1000 * dt, "steps": steps,
+            "h2d_bytes_per_step": int(12 * R.N), "d2h_bytes_per_step": 8,
+            "what": "per step: mf_train_epoch in out-of-core mode (staged=1: the epoch's ratings "
+                    "copied from pinned host memory, overlapped with compute) + mf_rmse (D2H); "
+                    "host wall clock",
+            "cold": {"value": R.N / dc, "unit": "updates/s", "ms_per_step": 1000 * dc,
+                     "h2d_bytes_per_step": int(12 * (R.N + R.Ntest)), "d2h_bytes_per_step": 8,
+                     "what": "per step: mf_create + mf_load_coo(train,test from pinned host; the "
+                             "whole one-time GPU preprocessing) + 1 epoch + mf_rmse"}}
 
 
 def ncu_traffic(args):

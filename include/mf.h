@@ -120,11 +120,6 @@ typedef struct mf_params {
                              each launch is exactly what one of G GPUs runs in that sub-epoch
                              (tools/scale_emulation.py).  Same result either way: a stratum's
                              blocks touch disjoint P and Q rows                                 */
-  int32_t q_atomic;       /* Hogwild q_v write: 0 = plain store of q' (the paper's GPU kernel),
-                             1 = L2 atomic add of q' - q (Hogwild!'s own component-wise atomic
-                             rule, ref [44]).  With one worker both give the same
-                             result; under concurrency the atomic rule loses no update of a hot
-                             column and runs hot rows faster.  Not with ADAGRAD.    */
 } mf_params;
 
 /* Fill *p with defaults (Table 3 Netflix lambda/alpha/beta, k = 128, fp32, Hogwild, f = 256). */

@@ -664,8 +664,6 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
     return MF_E_INVAL;
   if (p->prefetch < 0 || p->prefetch > 2) return MF_E_INVAL;
   if (p->wf_kernel < 0 || p->wf_kernel > 2 || p->launch_blocks < 0) return MF_E_INVAL;
-  if (p->q_atomic < 0 || p->q_atomic > 1) return MF_E_INVAL;
-  if (p->q_atomic && p->lr_rule == 1) return MF_E_UNSUPPORTED;
   if (p->transport < 0 || p->transport > 1) return MF_E_INVAL;
   if (p->staged < 0 || p->staged > 1) return MF_E_INVAL;
   if (p->lr_rule < 0 || p->lr_rule > 1 || !(p->ada_eps >= 0.f)) return MF_E_INVAL;
@@ -1378,7 +1376,6 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
     L.ada = ada_args(c);
     if (L.ada.GP) L.g = c->p.alpha;        // ADAGRAD: constant alpha, no Eq. 9 decay
-    L.qred = c->p.q_atomic;
     L.out_workers = &c->last_workers; L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
     CUDA_TRY(c, launch_hogwild(L));

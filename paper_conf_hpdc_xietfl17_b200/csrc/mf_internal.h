@@ -40,7 +40,6 @@ struct HogwildLaunch {
   void *P, *Q;
   float g, lp, lq;
   AdaArgs ada;              // ada.GP != nullptr: ADAGRAD (g = alpha)
-  int qred;                 // 1: q_v written as an L2 atomic add of the delta (Hogwild! [44])
   cudaStream_t stream;
   int *out_workers, *out_lanes, *out_grid;
 };

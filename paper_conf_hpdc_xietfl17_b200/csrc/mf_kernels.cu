@@ -23,7 +23,7 @@ constexpr int ring_ahead(int K, int S) { return ring_slots(K, S) == 32 ? 15 : 7;
 // f consecutive slots of its chunk serially.  Persistent grid: workers loop until the list is
 // exhausted.  The chunk list of a launch is the concatenation of up to kMaxSegs block segments.
 // ---------------------------------------------------------------------------------------------
-template <typename T, int K, int L, int D, bool ADA, bool QRED>
+template <typename T, int K, int L, int D, bool ADA>
 __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slots,
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
                                                  unsigned long long* __restrict__ counter,
@@ -56,8 +56,8 @@ __global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slot
       lo = (int64_t)chunk * f + segs.shift[sgi];
     }
     // every group of the warp runs f iterations in lockstep (inactive ones on sentinels)
-    run_serial<T, K, L, D, true, ADA, QRED>(slots, lo, f, act, P, Q, g, cp, cq, gl, gbase,
-                                            0xffffffffu, ada);
+    run_serial<T, K, L, D, true, ADA>(slots, lo, f, act, P, Q, g, cp, cq, gl, gbase, 0xffffffffu,
+                                      ada);
   }
 }
 
@@ -309,9 +309,9 @@ __global__ void k_rmse_final(const double* __restrict__ partial, int n, double* 
 // ---------------------------------------------------------------------------------------------
 // Dispatch
 // ---------------------------------------------------------------------------------------------
-template <typename T, int K, int L, int D, bool ADA = false, bool QRED = false>
+template <typename T, int K, int L, int D, bool ADA = false>
 static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
-  auto kern = k_hogwild<T, K, L, D, ADA, QRED>;
+  auto kern = k_hogwild<T, K, L, D, ADA>;
   const int threads = 256;
   int per_sm = 0;
   cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, 0);
@@ -431,7 +431,6 @@ template <typename T, int K, int LB>
 static cudaError_t hogwild_kl(const HogwildLaunch& a) {
   constexpr int S = (int)sizeof(T);
   if (a.ada.GP) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, true>(a);
-  if (a.qred) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, true>(a);
   if (a.prefetch == 1) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1>(a);
   return launch_hogwild_t<T, K, lanes_for(K, S, LB), 2>(a);
 }

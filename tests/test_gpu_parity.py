@@ -29,7 +29,7 @@ def pair(R, k=16, **kw):
     if R.ut is not None:
         g.load(R.ut, R.vt, R.rt, "test")
     okw = {kk: vv for kk, vv in kw.items() if kk not in ("lane_bytes", "prefetch", "wf_kernel", "staged",
-                                                          "launch_blocks", "q_atomic")}
+                                                          "launch_blocks")}
     if kw.get("schedule") == "wavefront":
         okw.setdefault("workers", kw.get("workers"))
     o = po.Oracle(R.m, R.n, k, R.u, R.v, R.r, **okw)
@@ -93,8 +93,6 @@ DET_CASES = [
     dict(schedule="hogwild", workers=1, grid_a=4, batch_f=16),
     dict(schedule="hogwild", workers=1, lane_bytes=32),
     dict(schedule="hogwild", workers=1, prefetch=2),
-    dict(schedule="hogwild", workers=1, q_atomic=True),
-    dict(schedule="hogwild", workers=1, q_atomic=True, grid_a=8, batch_f=64, launch_blocks=2),
 ]
 
 
@@ -169,10 +167,9 @@ def test_wavefront_is_deterministic_run_to_run():
 # exactly as the paper reports for Hugewiki with j = 4.  So the small-set tests run within
 # the rule; tests/test_gpu_fullsize.py checks full concurrency at Netflix scale.
 
-@pytest.mark.parametrize("storage,tol,qa", [("fp32", 0.005, False), ("fp16", 0.01, False),
-                                           ("fp32", 0.005, True), ("fp16", 0.01, True)])
-def test_hogwild_20_epoch_rmse_within_tolerance(tiny, storage, tol, qa):
-    g, o = pair(tiny, storage=storage, schedule="hogwild", workers=4, q_atomic=qa, **TABLE3_NETFLIX)
+@pytest.mark.parametrize("storage,tol", [("fp32", 0.005), ("fp16", 0.01)])
+def test_hogwild_20_epoch_rmse_within_tolerance(tiny, storage, tol):
+    g, o = pair(tiny, storage=storage, schedule="hogwild", workers=4, **TABLE3_NETFLIX)
     for _ in range(20):
         g.train_epoch()
         o.train_epoch()
@@ -180,15 +177,13 @@ def test_hogwild_20_epoch_rmse_within_tolerance(tiny, storage, tol, qa):
     assert abs(rg - ro) <= tol * ro, (rg, ro)
 
 
-@pytest.mark.parametrize("qa", [False, True])
-def test_hogwild_powerlaw_20_epochs_matches_oracle(qa):
+def test_hogwild_powerlaw_20_epochs_matches_oracle():
     """Skewed (power-law) data, n = 900, 32 concurrent workers (< n/20 = 45): collisions on hot
-    columns happen, and the 20-epoch RMSE still lands within 0.5% of the serial oracle (with
-    the plain-store and the atomic-delta q_v write)."""
+    columns happen, and the 20-epoch RMSE still lands within 0.5% of the serial oracle."""
     R = synth.powerlaw(4000, 900, 200_000, 20_000, seed=5, rank=8, mu=3.6, noise=0.5)
     R = synth.Ratings(R.m, R.n, R.u.numpy(), R.v.numpy(), R.r.numpy(), R.ut.numpy(), R.vt.numpy(),
                       R.rt.numpy())
-    g, o = pair(R, k=32, schedule="hogwild", workers=32, q_atomic=qa, **TABLE3_NETFLIX)
+    g, o = pair(R, k=32, schedule="hogwild", workers=32, **TABLE3_NETFLIX)
     for _ in range(20):
         g.train_epoch()
         o.train_epoch()
@@ -206,31 +201,6 @@ def test_hogwild_one_worker_reproduces_oracle_curve(tiny):
         o.train_epoch()
         rg, ro = g.rmse(), o.rmse(tiny.ut, tiny.vt, tiny.rt)
         assert abs(rg - ro) <= (1e-5 if t == 0 else 1e-4) * ro, (t, rg, ro)
-
-
-@pytest.mark.parametrize("storage", ["fp16", "bf16"])
-def test_hogwild_atomic_delta_one_worker_near_store(tiny, storage):
-    """One worker: the atomic-delta write adds d = RN(q') - q (both storage values) in L2.  d is
-    exact, and the row lands on RN(q') exactly, whenever q' and q are within a factor 2 of each
-    other (Sterbenz); near a sign change d rounds, giving a one-ulp offset that later updates
-    carry along (as in the fp16 wavefront bar).  Bar after one epoch: >75% of entries identical
-    to the plain-store run, all within 2 ulps of the largest binade, RMSE within 1e-4."""
-    outs = []
-    for qa in (False, True):
-        g = mf.MF(tiny.m, tiny.n, 16, schedule="hogwild", workers=1, storage=storage, q_atomic=qa,
-                  **TABLE3_NETFLIX)
-        g.load(tiny.u, tiny.v, tiny.r)
-        g.load(tiny.ut, tiny.vt, tiny.rt, "test")
-        g.train_epoch()
-        outs.append((g.factors(), g.rmse()))
-    (Ps, Qs), rs = outs[0]
-    (Pa, Qa), ra = outs[1]
-    mant = 10 if storage == "fp16" else 7
-    for Xs, Xa in ((Ps, Pa), (Qs, Qa)):
-        ulp_abs = 2.0 ** (np.floor(np.log2(np.abs(Xs).max())) - mant)
-        assert np.mean(Xs == Xa) > 0.75, float(np.mean(Xs == Xa))
-        assert np.abs(Xs - Xa).max() <= 2 * ulp_abs
-    assert abs(rs - ra) <= 1e-4 * rs
 
 
 def test_hogwild_epoch_updates_every_sample_once(tiny):

@@ -25,7 +25,6 @@ ap.add_argument("--storage", default="fp16")
 ap.add_argument("--workers", default="0")
 ap.add_argument("--mu", type=float, default=0.0)
 ap.add_argument("--epochs", type=int, default=4)
-ap.add_argument("--q-atomic", default="0", help="comma list of q_atomic settings (0, 1)")
 args = ap.parse_args()
 
 for n in [int(x) for x in args.ns.split(",")]:
@@ -34,9 +33,9 @@ for n in [int(x) for x in args.ns.split(",")]:
                            device="cuda")
         dv = torch.bincount(R.v.long(), minlength=n)
         top = float(dv.max()) / R.N
-        for w, qa in [(int(x), int(y)) for x in args.workers.split(",") for y in args.q_atomic.split(",")]:
+        for w in [int(x) for x in args.workers.split(",")]:
             g = mf.MF(R.m, R.n, 128, storage=args.storage, workers=w, lambda_p=0.03, alpha=0.08,
-                      beta=0.3, seed=42, q_atomic=bool(qa))
+                      beta=0.3, seed=42)
             g.load(R.u, R.v, R.r)
             g.load(R.ut, R.vt, R.rt, "test")
             curve, ms = [round(g.rmse(), 4)], []
@@ -45,7 +44,7 @@ for n in [int(x) for x in args.ns.split(",")]:
                 st = g.stats()
                 ms.append(st["sgd_ms"])
                 curve.append(round(g.rmse(), 4))
-            print(json.dumps(dict(n=n, a_v=a_v, top_col_share=round(top, 5), workers=st["workers"], q_atomic=qa,
+            print(json.dumps(dict(n=n, a_v=a_v, top_col_share=round(top, 5), workers=st["workers"],
                                   ms=round(float(np.median(ms[1:])), 3),
                                   gups=round(R.N / float(np.median(ms[1:])) / 1e6, 3),
                                   rmse=curve)), flush=True)

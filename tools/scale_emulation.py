@@ -34,7 +34,6 @@ ap.add_argument("--out", default=None)
 ap.add_argument("--gs", default="1,2,4,8", help="GPU counts to emulate")
 ap.add_argument("--workers", default="0", help="comma list of Hogwild worker counts (0 = all resident)")
 ap.add_argument("--no-base", action="store_true")
-ap.add_argument("--q-atomic", action="store_true")
 args = ap.parse_args()
 
 s = synth.SHAPES[args.workload]
@@ -47,7 +46,7 @@ t_comm = 20e-3 + msg / 770e9 * 1e3          # ms per sub-epoch
 
 
 def run(**kw):
-    g = mf.MF(R.m, R.n, K, storage=args.storage, seed=42, q_atomic=args.q_atomic, **hp, **kw)
+    g = mf.MF(R.m, R.n, K, storage=args.storage, seed=42, **hp, **kw)
     g.load(R.u, R.v, R.r)
     g.load(R.ut, R.vt, R.rt, "test")
     g.train_epoch()                          # warm-up
