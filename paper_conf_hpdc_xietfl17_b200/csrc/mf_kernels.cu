@@ -153,16 +153,56 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
   const float cp = 1.f - g * lp, cq = 1.f - g * lq;
   const int32_t* my_seq = seq + (int64_t)worker * c;
   const int32_t* my_rank = rank + (int64_t)worker * c;
+  const int64_t* my_off = sub_off + (int64_t)worker * c;
+  // Cross-wave pipeline: a wave's own work is ~20 samples, so its start-up chain (column id ->
+  // sub-block offsets -> ratings -> rows, plus the ticket poll) would otherwise cost several
+  // dependent memory round trips per wave.  While wave w runs, the next waves' inputs are in
+  // flight: column ids and ticket ranks 3 ahead, sub-block offsets 2 ahead, the first rating
+  // batches and a poll of the column ticket 1 ahead.  Only the rows (which the ticket guards)
+  // are read after the acquire.
+  auto col_at = [&](int w) { return w < c ? __ldg(my_seq + w) : 0; };
+  auto tgt_at = [&](int w) { return w < c ? __ldg(my_rank + w) : 0; };
+  int col0 = col_at(0), tgt0 = tgt_at(0);
+  int col1 = col_at(1), tgt1 = tgt_at(1);
+  int col2 = col_at(2), tgt2 = tgt_at(2);
+  int64_t lo0 = __ldg(my_off + col0) + shift;
+  int n0 = (int)(__ldg(my_off + col0 + 1) + shift - lo0);
+  int64_t lo1 = 0;
+  int n1 = 0;
+  if (c > 1) {
+    lo1 = __ldg(my_off + col1) + shift;
+    n1 = (int)(__ldg(my_off + col1 + 1) + shift - lo1);
+  }
+  RingHead h0 = load_head<L>(slots, dup, lo0, n0, gl);
+  int poll = ld_relaxed(tickets + col0);
   for (int w = 0; w < c; ++w) {
-    const int col = __ldg(my_seq + w);
-    const int tgt = __ldg(my_rank + w);
-    const int64_t sb = (int64_t)worker * c + col;
-    const int64_t lo = __ldg(sub_off + sb) + shift;
-    const int n = (int)(__ldg(sub_off + sb + 1) + shift - lo);
-    ticket_acquire(tickets + col, tgt);     // (empty sub-blocks still keep the visit order)
-    if (n > 0)
-      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo, n, P, Q, g, cp, cq, gl, gbase, gmask, ring);
-    ticket_release(tickets + col, tgt + 1, gmask, gl);
+    // acquire column col0: the poll (a relaxed load issued a wave ago) or a spin, then a fence
+    // unless the previous wave's release fence already follows the poll (acquire pattern:
+    // relaxed load, then fence.acq_rel, in program order)
+    if (poll != tgt0) {
+      ticket_acquire(tickets + col0, tgt0);
+    } else if (w == 0) {
+      fence_acq_rel();
+    }
+    // next waves' inputs
+    RingHead h1{};
+    if (w + 1 < c) h1 = load_head<L>(slots, dup, lo1, n1, gl);
+    int64_t lo2 = 0;
+    int n2 = 0;
+    if (w + 2 < c) {
+      lo2 = __ldg(my_off + col2) + shift;
+      n2 = (int)(__ldg(my_off + col2 + 1) + shift - lo2);
+    }
+    const int col3 = col_at(w + 3), tgt3 = tgt_at(w + 3);
+    const int poll1 = w + 1 < c ? ld_relaxed(tickets + col1) : 0;
+    if (n0 > 0)
+      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo0, n0, h0, P, Q, g, cp, cq, gl, gbase, gmask,
+                                        ring);
+    ticket_release(tickets + col0, tgt0 + 1, gmask, gl);   // fence; syncwarp; relaxed store
+    poll = poll1;
+    col0 = col1; tgt0 = tgt1; lo0 = lo1; n0 = n1; h0 = h1;
+    col1 = col2; tgt1 = tgt2; lo1 = lo2; n1 = n2;
+    col2 = col3; tgt2 = tgt3;
   }
 }
 

@@ -107,3 +107,28 @@ def test_fullsize_wavefront_deterministic_rerun(netflix):
         outs.append(g.factors())
         g.close()
     assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+
+
+def test_bench_deterministic_config_oracle_parity_at_scale():
+    """The deterministic line's exact launch configuration (fp32, k = 128, s = 768 workers,
+    c = 6144 column blocks, cyclic order) on a Netflix-shaped set large enough that n >= c
+    (35% scale: 34.7 M ratings, 168 K x 6.2 K), one epoch, against the oracle's serial (w, i)
+    loop element by element: |dP|, |dQ| <= 1e-4 and test RMSE within 1e-5 (north_star)."""
+    R = synth.shaped("netflix", fraction=0.35, device="cuda")
+    assert R.n >= 6144
+    kw = dict(storage="fp32", schedule="wavefront", workers=768, wf_cols=6144, cyclic=True,
+              seed=SEED, **HP)
+    g = mf.MF(R.m, R.n, 128, **kw)
+    g.load(R.u, R.v, R.r)
+    g.load(R.ut, R.vt, R.rt, "test")
+    g.train_epoch()
+    Pg, Qg = g.factors()
+    rg = g.rmse()
+    g.close()
+    h = [x.cpu().numpy() for x in (R.u, R.v, R.r, R.ut, R.vt, R.rt)]
+    o = po.Oracle(R.m, R.n, 128, h[0], h[1], h[2], **kw)
+    o.train_epoch()
+    Po, Qo = o.factors()
+    ro = o.rmse(h[3], h[4], h[5])
+    assert np.abs(Pg - Po).max() <= 1e-4 and np.abs(Qg - Qo).max() <= 1e-4
+    assert abs(rg - ro) <= 1e-5 * ro, (rg, ro)
