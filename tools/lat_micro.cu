@@ -80,6 +80,24 @@ __global__ void k_chain(float* out, long long* cyc, float seed) {
   }
   t1 = clock64();
   if (l == 0) cyc[5] = t1 - t0;
+  // 7. integer warp reduction (REDUX.SUM) chained
+  int xi = (int)x;
+  t0 = clock64();
+#pragma unroll 16
+  for (int i = 0; i < IT; ++i) xi = __reduce_add_sync(~0u, xi) >> 5;
+  t1 = clock64();
+  if (l == 0) cyc[6] = t1 - t0;
+  x += xi;
+  // 8. fixed-point all-reduce: F2I (scale 2^24) + REDUX.SUM + I2F, chained
+  t0 = clock64();
+#pragma unroll 4
+  for (int i = 0; i < IT / 8; ++i) {
+    const int q = __float2int_rn(x * 16777216.f);
+    const float s = (float)__reduce_add_sync(~0u, q) * (1.f / 16777216.f);
+    x = x * 0.5f + s * 1e-3f;
+  }
+  t1 = clock64();
+  if (l == 0) cyc[7] = t1 - t0;
   out[l] = x;
 }
 
@@ -87,7 +105,7 @@ int main() {
   float* out;
   long long* cyc;
   cudaMalloc(&out, 32 * 4);
-  cudaMallocManaged(&cyc, 8 * 8);
+  cudaMallocManaged(&cyc, 16 * 8);
   for (int rep = 0; rep < 2; ++rep) {
     k_chain<<<1, 32>>>(out, cyc, 1.0f);
     cudaDeviceSynchronize();
@@ -98,5 +116,7 @@ int main() {
   printf("bfly32 allreduce %.1f cyc (+2 fp)\n", (double)cyc[3] / (IT / 8));
   printf("smem allreduce   %.1f cyc (+2 fp)\n", (double)cyc[4] / (IT / 8));
   printf("bfly16 allreduce %.1f cyc (+2 fp)\n", (double)cyc[5] / (IT / 8));
+  printf("redux.add.s32    %.1f cyc (+1 shift)\n", (double)cyc[6] / IT);
+  printf("fixed-pt redux   %.1f cyc (+2 fp)\n", (double)cyc[7] / (IT / 8));
   return 0;
 }
