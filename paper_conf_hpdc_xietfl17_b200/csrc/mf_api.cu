@@ -10,6 +10,8 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <cstdlib>
+#include <map>
 #include <cub/cub.cuh>
 #include <string>
 #include <vector>
@@ -1401,8 +1403,45 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     L.ada = ada_args(c);
     if (L.ada.GP) L.g = c->p.alpha;
     L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
+    // Diagnostics only (MF_PROFILE_WAVES=1): per-worker clock64 totals of ticket waits and
+    // sub-block runs, summarised on stderr after the launch (synchronises).
+    static const bool kProfWaves = std::getenv("MF_PROFILE_WAVES") != nullptr;
+    long long* prof = nullptr;
+    if (kProfWaves && L.variant == 1) {
+      CUDA_TRY(c, cudaMallocAsync(reinterpret_cast<void**>(&prof), (size_t)c->s * 6 * 8, c->st));
+      CUDA_TRY(c, cudaMemsetAsync(prof, 0, (size_t)c->s * 6 * 8, c->st));
+    }
+    L.prof = prof;
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
     cudaError_t e = launch_wavefront(L);
+    if (prof && e == cudaSuccess) {
+      std::vector<long long> h((size_t)c->s * 6);
+      CUDA_TRY(c, cudaMemcpyAsync(h.data(), prof, h.size() * 8, cudaMemcpyDeviceToHost, c->st));
+      CUDA_TRY(c, cudaStreamSynchronize(c->st));
+      CUDA_TRY(c, cudaFreeAsync(prof, c->st));
+      std::map<long long, int> per_smsp;
+      for (int i = 0; i < c->s; ++i) ++per_smsp[h[6 * i + 3] * 4 + (h[6 * i + 4] & 3)];
+      double sw = 0, sr = 0, mxw = 0, mxr = 0, mxt = 0, sn = 0, shared_r = 0, solo_r = 0;
+      double shared_n = 0, solo_n = 0, srel = 0;
+      for (int i = 0; i < c->s; ++i) {
+        const double w = (double)h[6 * i], r = (double)h[6 * i + 1], n = (double)h[6 * i + 2];
+        srel += (double)h[6 * i + 5];
+        sw += w; sr += r; sn += n;
+        mxw = std::max(mxw, w); mxr = std::max(mxr, r); mxt = std::max(mxt, w + r);
+        const bool shared = per_smsp[h[6 * i + 3] * 4 + (h[6 * i + 4] & 3)] > 1;
+        (shared ? shared_r : solo_r) += r;
+        (shared ? shared_n : solo_n) += n;
+      }
+      int shared_w = 0;
+      for (auto& kv : per_smsp) if (kv.second > 1) shared_w += kv.second;
+      std::fprintf(stderr,
+                   "[MF_PROFILE_WAVES] s=%d c=%d  cycles/worker: wait mean %.3g max %.3g, run mean %.3g "
+                   "max %.3g, wait+run max %.3g; run cycles/sample %.1f (solo-SMSP workers %.1f, "
+                   "SMSP-sharing %.1f; %d of %d workers share an SMSP); release fence mean %.3g cycles/worker\n",
+                   c->s, c->c, sw / c->s, mxw, sr / c->s, mxr, mxt, sr / std::max(sn, 1.0),
+                   solo_r / std::max(solo_n, 1.0), shared_r / std::max(shared_n, 1.0), shared_w, c->s,
+                   srel / c->s);
+    }
     if (e == cudaErrorCooperativeLaunchTooLarge) {
       cudaGetLastError();
       return c->fail(MF_E_UNSUPPORTED, "wavefront: %d workers cannot all be co-resident", c->s);

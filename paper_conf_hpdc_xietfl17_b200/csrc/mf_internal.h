@@ -59,6 +59,8 @@ struct WavefrontLaunch {
   void *P, *Q;
   float g, lp, lq;
   AdaArgs ada;              // ada.GP != nullptr: ADAGRAD (register kernel; g = alpha)
+  long long* prof;          // diagnostics (MF_PROFILE_WAVES): per worker {wait, run, samples, smid, warpid, release
+                            // fence} clock64 totals, or nullptr
   cudaStream_t stream;
   int *out_lanes, *out_grid;
 };

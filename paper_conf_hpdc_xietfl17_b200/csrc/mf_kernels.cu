@@ -77,6 +77,11 @@ __device__ __forceinline__ int ld_relaxed(const int* p) {
 __device__ __forceinline__ void st_relaxed(int* p, int v) {
   asm volatile("st.relaxed.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
+__device__ __forceinline__ int ld_acquire(const int* p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
 __device__ __forceinline__ void fence_acq_rel() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 
 // Acquire the column: spin with RELAXED loads (an ld.acquire per poll would emit an L1
@@ -137,7 +142,8 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
                                                     const int32_t* __restrict__ rank,
                                                     int* __restrict__ tickets, int s, int c,
                                                     T* __restrict__ P, T* __restrict__ Q, float g,
-                                                    float lp, float lq, int64_t shift) {
+                                                    float lp, float lq, int64_t shift,
+                                                    long long* __restrict__ prof) {
   extern __shared__ __align__(16) char smem[];
   constexpr int ROWB = K * (int)sizeof(T);
   const int lane = threadIdx.x & 31;
@@ -158,8 +164,11 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
   // sub-block offsets -> ratings -> rows, plus the ticket poll) would otherwise cost several
   // dependent memory round trips per wave.  While wave w runs, the next waves' inputs are in
   // flight: column ids and ticket ranks 3 ahead, sub-block offsets 2 ahead, the first rating
-  // batches and a poll of the column ticket 1 ahead.  Only the rows (which the ticket guards)
-  // are read after the acquire.
+  // batches and an ld.acquire of the column ticket 1 ahead.  The rows (which the ticket guards)
+  // are read only after an acquire: when the early ld.acquire already shows the ticket, the
+  // next sub-block's first F+1 rows are prefetched before this wave's release fence, so the
+  // fence's wait and their memory latency overlap (MF_PROFILE_WAVES: the release fence is
+  // ~2,800 cycles per wave, a quarter of the epoch).
   auto col_at = [&](int w) { return w < c ? __ldg(my_seq + w) : 0; };
   auto tgt_at = [&](int w) { return w < c ? __ldg(my_rank + w) : 0; };
   int col0 = col_at(0), tgt0 = tgt_at(0);
@@ -174,15 +183,15 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     n1 = (int)(__ldg(my_off + col1 + 1) + shift - lo1);
   }
   RingHead h0 = load_head<L>(slots, dup, lo0, n0, gl);
-  int poll = ld_relaxed(tickets + col0);
+  bool ready = false;            // column col0 acquired and its ring prologue issued already
+  long long t_wait = 0, t_run = 0, t_rel = 0, n_done = 0;
   for (int w = 0; w < c; ++w) {
-    // acquire column col0: the poll (a relaxed load issued a wave ago) or a spin, then a fence
-    // unless the previous wave's release fence already follows the poll (acquire pattern:
-    // relaxed load, then fence.acq_rel, in program order)
-    if (poll != tgt0) {
-      ticket_acquire(tickets + col0, tgt0);
-    } else if (w == 0) {
-      fence_acq_rel();
+    const long long tw0 = prof ? clock64() : 0;
+    if (!ready) {
+      ticket_acquire(tickets + col0, tgt0);   // relaxed spin + fence.acq_rel
+      if (n0 > 0)
+        run_subblock_ring<T, K, L, RS, F>(slots, dup, lo0, n0, h0, P, Q, g, cp, cq, gl, gbase,
+                                          gmask, ring, true, false);
     }
     // next waves' inputs
     RingHead h1{};
@@ -194,15 +203,37 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
       n2 = (int)(__ldg(my_off + col2 + 1) + shift - lo2);
     }
     const int col3 = col_at(w + 3), tgt3 = tgt_at(w + 3);
-    const int poll1 = w + 1 < c ? ld_relaxed(tickets + col1) : 0;
+    // early acquire attempt for the next column: an ld.acquire, so if it already shows the
+    // ticket the next sub-block's rows may be read from here on (program order)
+    const int poll1 = w + 1 < c ? ld_acquire(tickets + col1) : -1;
+    const long long tw1 = prof ? clock64() : 0;
     if (n0 > 0)
       run_subblock_ring<T, K, L, RS, F>(slots, dup, lo0, n0, h0, P, Q, g, cp, cq, gl, gbase, gmask,
-                                        ring);
+                                        ring, false, true);
+    // next column already released: issue its row prefetch BEFORE this wave's release fence.
+    // (Its p rows may have been stored by this sub-block: same thread, issued after them.)
+    ready = w + 1 < c && poll1 == tgt1;
+    if (ready && n1 > 0)
+      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo1, n1, h1, P, Q, g, cp, cq, gl, gbase, gmask,
+                                        ring, true, false);
+    const long long tw2 = prof ? clock64() : 0;
     ticket_release(tickets + col0, tgt0 + 1, gmask, gl);   // fence; syncwarp; relaxed store
-    poll = poll1;
+    if (prof) {
+      t_wait += tw1 - tw0;
+      t_run += tw2 - tw1;
+      t_rel += clock64() - tw2;
+      n_done += n0;
+    }
     col0 = col1; tgt0 = tgt1; lo0 = lo1; n0 = n1; h0 = h1;
     col1 = col2; tgt1 = tgt2; lo1 = lo2; n1 = n2;
     col2 = col3; tgt2 = tgt3;
+  }
+  if (prof && gl == 0) {
+    unsigned smid, wid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    asm volatile("mov.u32 %0, %%warpid;" : "=r"(wid));
+    long long* o = prof + 6 * (int64_t)worker;
+    o[0] = t_wait; o[1] = t_run; o[2] = n_done; o[3] = smid; o[4] = wid; o[5] = t_rel;
   }
 }
 
@@ -429,8 +460,9 @@ static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
   T* Q = reinterpret_cast<T*>(a.Q);
   float g = a.g, lp = a.lp, lq = a.lq;
   int64_t shift = a.shift;
+  long long* prof = a.prof;
   void* args[] = {&slots, &dup, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq,
-                  &shift};
+                  &shift, &prof};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, smem,
                                      a.stream);
 }
