@@ -91,7 +91,9 @@ typedef struct mf_params {
   int32_t grid_a;         /* strata grid a x a (0 = 1 if world == 1 else 8); a % world == 0
                              and a / world <= 16                                                */
   int32_t cyclic;         /* wavefront: 1 = cyclic column order (A: cyclic variant), needs c >= s */
-  int32_t lane_bytes;     /* Hogwild/RMSE kernel: bytes of p_u (and q_v) per lane, 16 or 32 (0 = 16) */
+  int32_t lane_bytes;     /* Hogwild/RMSE kernel: bytes of p_u (and q_v) per lane, 16 or 32 (0 = 16).
+                             Ring wavefront: 0 = default geometry (fp16/bf16 k = 128: 8 B on 32
+                             lanes), 16 = 16-B lanes, 32 / 64 = half / quarter of the lanes   */
   int32_t prefetch;       /* Hogwild software-pipeline depth: samples in flight per worker, 1 or 2 (0 = 1) */
   int32_t lr_rule;        /* 0 = Eq. 9 schedule (the paper); 1 = ADAGRAD (P:L419 future work,
                              Duchi et al. [20]; R23): per-coordinate fp32 accumulators

@@ -15,6 +15,12 @@ constexpr int ring_slots(int K, int S) {
   return (32 * 2 * K * S <= 32768 && ring_lanes(K, S) > 15) ? 32 : 16;
 }
 constexpr int ring_ahead(int K, int S) { return ring_slots(K, S) == 32 ? 15 : 7; }
+// Narrow-slice full-warp ring (default for k*S = 128 or 256 bytes): 32 lanes of 4 or 8 B
+// (cp.async.ca row copies), RS = 32, F = 15 -- the full-batch RS == L path and the
+// integer-reduction group sum of the 32-lane geometry.
+constexpr bool narrow_ring(int K, int S) { return K * S == 128 || K * S == 256; }
+// 64-byte rows (fp16 k = 32, fp32 k = 16): 16 lanes of 4 B, RS = 16, F = 7 (RS == L again).
+constexpr bool narrow16_ring(int K, int S) { return K * S == 64; }
 
 // ---------------------------------------------------------------------------------------------
 // batch-Hogwild! (section 5.1).  A worker is a group of L lanes; a warp holds
@@ -532,6 +538,11 @@ static cudaError_t wavefront_k(const WavefrontLaunch& a) {
   constexpr int L4 = L2 / 4;                 // lane_bytes = 64: a quarter of the lanes
   if constexpr (quarter_ring_ok(K, S))
     if (a.variant == 1 && a.dup && a.lane_bytes == 64) return launch_wavefront2_t<T, K, L4, 16, 7>(a);
+  // narrow slices on a full warp (lane_bytes = 0); lane_bytes = 16 keeps 16-B lanes
+  if constexpr (narrow_ring(K, S))
+    if (a.variant == 1 && a.dup && a.lane_bytes == 0) return launch_wavefront2_t<T, K, 32, 32, 15>(a);
+  if constexpr (narrow16_ring(K, S))
+    if (a.variant == 1 && a.dup && a.lane_bytes == 0) return launch_wavefront2_t<T, K, 16, 16, 7>(a);
   if constexpr (L2 > ring_ahead(K, S) && (K * S / L2) % 16 == 0)  // needs F < L, 16-B pieces
     if (a.variant == 1 && a.dup) return launch_wavefront2_t<T, K, L2>(a);
   return launch_wavefront_t<T, K, lanes_for(K, S, 8)>(a);
@@ -576,6 +587,8 @@ cudaError_t launch_libmf(const LibmfLaunch& a) { MF_DISPATCH(libmf_k, a) }
 template <int K, int S>
 static int ring_window_t(int lane_bytes) {
   if (lane_bytes == 64 && quarter_ring_ok(K, S)) return 16 - 7 - 1;  // RS = 16, F = 7
+  if (lane_bytes == 0 && narrow_ring(K, S)) return 32 - 15 - 1;        // RS = 32, F = 15
+  if (lane_bytes == 0 && narrow16_ring(K, S)) return 16 - 7 - 1;        // RS = 16, F = 7
   return ring_slots(K, S) - ring_ahead(K, S) - 1;
 }
 

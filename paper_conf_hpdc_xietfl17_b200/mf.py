@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libmf_b200.so")
+LIB_PATH = os.environ.get("MF_LIB", os.path.join(HERE, "libmf_b200.so"))   # MF_LIB: a variant build (tools/)
 
 STORAGE = {"fp32": 0, "fp16": 1, "bf16": 2}
 SCHEDULE = {"hogwild": 0, "wavefront": 1, "libmf": 2}

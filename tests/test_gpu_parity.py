@@ -125,19 +125,23 @@ def test_deterministic_parity_other_k_ragged(k, wfk, lb):
     assert abs(g.rmse() - o.rmse(R.ut, R.vt, R.rt)) <= 1e-5 * o.rmse(R.ut, R.vt, R.rt)
 
 
-@pytest.mark.parametrize("storage", ["fp16", "bf16"])
-def test_deterministic_parity_low_precision_storage(tiny, storage):
+@pytest.mark.parametrize("storage,k,lb", [("fp16", 16, 0), ("bf16", 16, 0), ("fp16", 128, 0),
+                                         ("bf16", 128, 0), ("fp16", 128, 16)])
+def test_deterministic_parity_low_precision_storage(tiny, storage, k, lb):
     """Storage rounding is RNE on both sides (R16), but the fp32 value being rounded
     differs between the two sides by the dot-product order (tree vs sequential, ~k*eps32), so an
     update can round to the neighbouring storage value: one ulp of that value's binade, which
     later updates carry along as an ABSOLUTE offset (damped by gamma).  Bar: every entry within
     2 ulps of the largest binade in use (absolute), >75% of entries identical, test RMSE within
-    1e-4 relative."""
-    g, o = pair(tiny, storage=storage, schedule="wavefront", workers=8, wf_cols=16, **TABLE3_NETFLIX)
+    1e-4 relative.  k = 128 runs the ring kernel on the ragged set: lb = 0
+    is its default 32-lane geometry (8-B lane slices, split row copy), lb = 16 the 16-lane one."""
+    R = tiny if k == 16 else ragged()
+    g, o = pair(R, k=k, storage=storage, schedule="wavefront", workers=8 if k == 16 else 6,
+                wf_cols=16 if k == 16 else 9, lane_bytes=lb, **TABLE3_NETFLIX)
     g.train_epoch()
     o.train_epoch()
     mant = 10 if storage == "fp16" else 7
-    rg, ro = g.rmse(), o.rmse(tiny.ut, tiny.vt, tiny.rt)
+    rg, ro = g.rmse(), o.rmse(R.ut, R.vt, R.rt)
     for Xg, Xo in zip(g.factors(), o.factors()):
         ulp_abs = 2.0 ** (np.floor(np.log2(np.abs(Xo).max())) - mant)
         diag = (storage, float(np.mean(Xg == Xo)), float(np.abs(Xg - Xo).max()), ulp_abs, rg, ro)

@@ -32,6 +32,24 @@ __device__ __forceinline__ unsigned smid() {
   return s;
 }
 
+// Latency of one ld.cg from this SM to *p: a chain of 32 dependent loads (the loaded value,
+// always 0, is added to the next address), closed by a shared-memory store of the result
+// before the clock read so the clock waits for the last load.
+__device__ __forceinline__ long long chain_lat(const unsigned* p, volatile unsigned* sink_smem) {
+  unsigned x = 0;
+  long long best = 1LL << 40;
+  for (int rep = 0; rep < 4; ++rep) {
+    const long long t0 = clock64();
+#pragma unroll
+    for (int i = 0; i < 32; ++i)
+      asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(x) : "l"(p + x) : "memory");
+    *sink_smem = x;
+    const long long t1 = clock64();
+    if (rep > 0 && t1 - t0 < best) best = t1 - t0;
+  }
+  return best / 32;
+}
+
 // One CTA per SM (forced by dynamic smem); thread 0 times dependent loads.
 __global__ void k_latency(const unsigned* __restrict__ base, int* out_smid, float* lat) {
   extern __shared__ char smem[];
@@ -39,23 +57,10 @@ __global__ void k_latency(const unsigned* __restrict__ base, int* out_smid, floa
   smem[0] = 0;
   const unsigned s = smid();
   out_smid[blockIdx.x] = (int)s;
-  unsigned dep = 0;
   for (int g = 0; g < NPROBE; ++g) {
     const unsigned* p = base + (size_t)g * (GRAN / 4) * 3;   // granules 3 apart
-    long long best = 1LL << 40;
-    for (int rep = 0; rep < 12; ++rep) {
-      const unsigned* q = p + (dep & 0);                      // dependent on the previous load
-      long long t0 = clock64();
-      unsigned x;
-      asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(x) : "l"(q) : "memory");
-      dep += x;
-      asm volatile("" ::"r"(dep));
-      long long t1 = clock64();
-      if (rep > 1) best = (t1 - t0 < best) ? (t1 - t0) : best;
-    }
-    lat[blockIdx.x * NPROBE + g] = (float)best;
+    lat[blockIdx.x * NPROBE + g] = (float)chain_lat(p, (volatile unsigned*)smem);
   }
-  if (dep == 0xdeadbeef) out_smid[0] = -1;
 }
 
 // Per-row latency from one SM: probes rows, returns best latency per row.
@@ -66,22 +71,8 @@ __global__ void k_row_latency(const uint4* __restrict__ rows, const int* __restr
   smem[0] = 0;
   if ((int)smid() != want_sm) return;
   *hit = 1;
-  unsigned dep = 0;
-  for (int r = 0; r < nrows; ++r) {
-    const unsigned* p = (const unsigned*)(rows + (size_t)row_ids[r] * 16);
-    long long best = 1LL << 40;
-    for (int rep = 0; rep < 12; ++rep) {
-      long long t0 = clock64();
-      unsigned x;
-      asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(x) : "l"(p + (dep & 0)) : "memory");
-      dep += x;
-      asm volatile("" ::"r"(dep));
-      long long t1 = clock64();
-      if (rep > 1) best = (t1 - t0 < best) ? (t1 - t0) : best;
-    }
-    lat[r] = (float)best;
-  }
-  if (dep == 0xdeadbeef) *hit = 2;
+  for (int r = 0; r < nrows; ++r)
+    lat[r] = (float)chain_lat((const unsigned*)(rows + (size_t)row_ids[r] * 16), (volatile unsigned*)smem);
 }
 
 // mode: 0 all, 1 only die-0 SMs (rows set A), 2 split (die d uses set d), 3 split-x
