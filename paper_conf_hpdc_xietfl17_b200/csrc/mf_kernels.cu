@@ -89,6 +89,9 @@ __device__ __forceinline__ int ld_acquire(const int* p) {
   return v;
 }
 __device__ __forceinline__ void fence_acq_rel() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+// Release-only fence (PTX 8.6+): MEMBAR.GPU without the L1 invalidate (CCTL.IVALL) of acq_rel;
+// a release needs only this thread's prior stores ordered before the ticket store.
+__device__ __forceinline__ void fence_release() { asm volatile("fence.release.gpu;" ::: "memory"); }
 
 // Acquire the column: spin with RELAXED loads (an ld.acquire per poll would emit an L1
 // invalidate each time and flood L2 with strong loads on the few ticket lines) and exponential
@@ -104,7 +107,7 @@ __device__ __forceinline__ void ticket_acquire(const int* t, int tgt) {
 // Release: every lane fences its own row stores, the group re-converges (memory ordering among
 // the participating lanes), and one lane publishes ticket+1 (fence + relaxed store = release).
 __device__ __forceinline__ void ticket_release(int* t, int next, unsigned gmask, int gl) {
-  fence_acq_rel();
+  fence_release();
   __syncwarp(gmask);
   if (gl == 0) st_relaxed(t, next);
 }
