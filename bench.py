@@ -330,12 +330,14 @@ def main():
 
 def run_deterministic(args, R, hp, stream):
     """The north_star target run: the deterministic conflict-free wavefront (oracle-exact
-    order), fp32 storage, k = args.k, s = 768 workers, cyclic column order with c = 8s
-    (SURVEY App. A cyclic variant), on the same data; device-timed like the main line."""
+    order), fp32 storage, k = args.k, s = 888 workers (all co-resident: 6 per SM at 32 KB of
+    ring each), cyclic column order with c = 7680 (SURVEY App. A cyclic variant; s and c from
+    the sweep in profiles/r01_wavefront_sweep.md), on the same data; device-timed like the main
+    line."""
     from paper_conf_hpdc_xietfl17_b200 import mf
     steps, warm = max(3, args.steps // 2), 2
-    m = mf.MF(R.m, R.n, args.k, stream=stream, schedule="wavefront", storage="fp32", workers=768,
-              wf_cols=6144, cyclic=True, seed=42, **hp)
+    m = mf.MF(R.m, R.n, args.k, stream=stream, schedule="wavefront", storage="fp32", workers=888,
+              wf_cols=7680, cyclic=True, seed=42, **hp)
     m.load(R.u, R.v, R.r, "train")
     m.load(R.ut, R.vt, R.rt, "test")
     for _ in range(warm):
@@ -356,7 +358,7 @@ def run_deterministic(args, R, hp, stream):
     hbm, _ = peaks()
     bpu = st["bytes_per_update"]
     achieved = upd * bpu / (float(np.sum(sgd)) / 1000.0) / 1e9
-    out = {"schedule": "wavefront (deterministic, cyclic, s=768, c=6144)", "storage": "fp32",
+    out = {"schedule": "wavefront (deterministic, cyclic, s=888, c=7680)", "storage": "fp32",
            "value": upd / (ms / 1000.0), "unit": "updates/s", "ms_per_step": ms / steps,
            "steps": steps, "warmup": warm, "test_rmse": m.rmse("test"),
            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",

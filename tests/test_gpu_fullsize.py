@@ -110,13 +110,13 @@ def test_fullsize_wavefront_deterministic_rerun(netflix):
 
 
 def test_bench_deterministic_config_oracle_parity_at_scale():
-    """The deterministic line's exact launch configuration (fp32, k = 128, s = 768 workers,
-    c = 6144 column blocks, cyclic order) on a Netflix-shaped set large enough that n >= c
-    (35% scale: 34.7 M ratings, 168 K x 6.2 K), one epoch, against the oracle's serial (w, i)
+    """The deterministic line's exact launch configuration (fp32, k = 128, s = 888 workers,
+    c = 7680 column blocks, cyclic order) on a Netflix-shaped set large enough that n >= c
+    (45% scale: 44.6 M ratings, 216 K x 8.0 K), one epoch, against the oracle's serial (w, i)
     loop element by element: |dP|, |dQ| <= 1e-4 and test RMSE within 1e-5 (north_star)."""
-    R = synth.shaped("netflix", fraction=0.35, device="cuda")
-    assert R.n >= 6144
-    kw = dict(storage="fp32", schedule="wavefront", workers=768, wf_cols=6144, cyclic=True,
+    R = synth.shaped("netflix", fraction=0.45, device="cuda")
+    assert R.n >= 7680
+    kw = dict(storage="fp32", schedule="wavefront", workers=888, wf_cols=7680, cyclic=True,
               seed=SEED, **HP)
     g = mf.MF(R.m, R.n, 128, **kw)
     g.load(R.u, R.v, R.r)
