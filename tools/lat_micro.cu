@@ -98,7 +98,49 @@ __global__ void k_chain(float* out, long long* cyc, float seed) {
   }
   t1 = clock64();
   if (l == 0) cyc[7] = t1 - t0;
-  out[l] = x;
+  // 9. the kernel's split fixed-point group sum (hi 2^-12 + lo 2^-36, two F2I, two REDUX)
+  t0 = clock64();
+#pragma unroll 4
+  for (int i = 0; i < IT / 8; ++i) {
+    const int hi = __float2int_rn(x * 4096.f);
+    const float rem = fmaf((float)hi, -1.f / 4096.f, x);
+    const int lo = __float2int_rn(rem * 68719476736.f);
+    const int shi = __reduce_add_sync(~0u, hi), slo = __reduce_add_sync(~0u, lo);
+    const float s = fmaf((float)shi, 1.f / 4096.f, (float)slo * (1.f / 68719476736.f));
+    x = x * 0.5f + s * 1e-3f;
+  }
+  t1 = clock64();
+  if (l == 0) cyc[8] = t1 - t0;
+  // 10. the same sum with magic-number rounding (FADD to 1.5*2^k) instead of F2I / I2F
+  t0 = clock64();
+#pragma unroll 4
+  for (int i = 0; i < IT / 8; ++i) {
+    const float M1 = 12582912.f * (1.f / 4096.f);          // 1.5*2^23 * 2^-12: ulp 2^-12
+    const float t = x + M1;                                 // RNE to a multiple of 2^-12
+    const int hi = __float_as_int(t) - __float_as_int(M1);  // that multiple, in units of 2^-12
+    const float rem = x - (t - M1);                         // exact
+    const float M2 = 12582912.f;                            // ulp 1
+    const float t2 = fmaf(rem, 68719476736.f, M2);          // rem*2^36 rounded to an integer
+    const int lo = __float_as_int(t2) - __float_as_int(M2);
+    const int shi = __reduce_add_sync(~0u, hi), slo = __reduce_add_sync(~0u, lo);
+    const float s = fmaf((float)shi, 1.f / 4096.f, (float)slo * (1.f / 68719476736.f));
+    x = x * 0.5f + s * 1e-3f;
+  }
+  t1 = clock64();
+  if (l == 0) cyc[9] = t1 - t0;
+  // 11. F2I.rn chain, 12. I2F chain
+  t0 = clock64();
+#pragma unroll 16
+  for (int i = 0; i < IT; ++i) xi = __float2int_rn((float)xi * 0.5f);
+  t1 = clock64();
+  if (l == 0) cyc[10] = t1 - t0;
+  x += xi;
+  t0 = clock64();
+#pragma unroll 16
+  for (int i = 0; i < IT; ++i) xi = (int)__int2float_rn(xi + 1) ;
+  t1 = clock64();
+  if (l == 0) cyc[11] = t1 - t0;
+  out[l] = x + xi;
 }
 
 int main() {
@@ -118,5 +160,9 @@ int main() {
   printf("bfly16 allreduce %.1f cyc (+2 fp)\n", (double)cyc[5] / (IT / 8));
   printf("redux.add.s32    %.1f cyc (+1 shift)\n", (double)cyc[6] / IT);
   printf("fixed-pt redux   %.1f cyc (+2 fp)\n", (double)cyc[7] / (IT / 8));
+  printf("split redux (kernel) %.1f cyc (+2 fp)\n", (double)cyc[8] / (IT / 8));
+  printf("split redux magic    %.1f cyc (+2 fp)\n", (double)cyc[9] / (IT / 8));
+  printf("f2i.rn+fmul chain    %.1f cyc\n", (double)cyc[10] / IT);
+  printf("i2f+f2i(trunc)+iadd  %.1f cyc\n", (double)cyc[11] / IT);
   return 0;
 }
