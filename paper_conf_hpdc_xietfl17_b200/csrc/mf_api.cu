@@ -332,6 +332,54 @@ __global__ void k_cyclic_seq(const int32_t* __restrict__ tau, const int32_t* __r
   }
 }
 
+// Cyclic variant, ticket ranks in closed form (no sort).  Worker i visits column
+// sigma[(tau[i] + w) mod c] in wave w, so the s visits of one column fall in distinct waves,
+// and the rank of visit (w, i) -- the number of earlier (w', i') visits of that column -- is
+// the number of workers i' whose offset lies in the cyclic window (tau[i], tau[i] + w].  With
+// P_b(y) = #{i' < s : tau_b[i'] < y} that is P(a+w+1) - P(a+1), or across the wrap
+// (P(c) - P(a+1)) + P(a+w-c+1), a = tau_b[i].
+// k_tau_prefix: one CTA per block b builds P_b(0..c) (occupancy of the first s offsets, then
+// an inclusive scan in place).
+__global__ void __launch_bounds__(1024) k_tau_prefix(const int32_t* __restrict__ tau, int s, int c,
+                                                     int32_t* __restrict__ P) {
+  __shared__ int32_t part[1024];
+  const int64_t b = blockIdx.x;
+  int32_t* Pb = P + b * (int64_t)(c + 1);
+  for (int y = threadIdx.x; y <= c; y += blockDim.x) Pb[y] = 0;
+  __syncthreads();
+  for (int i = threadIdx.x; i < s; i += blockDim.x) Pb[1 + tau[b * (int64_t)c + i]] = 1;
+  __syncthreads();
+  const int ch = (c + (int)blockDim.x - 1) / (int)blockDim.x;
+  const int lo = 1 + (int)threadIdx.x * ch, hi = min(c + 1, lo + ch);
+  int32_t sum = 0;
+  for (int y = lo; y < hi; ++y) sum += Pb[y];
+  part[threadIdx.x] = sum;
+  __syncthreads();
+  for (int o = 1; o < (int)blockDim.x; o <<= 1) {     // Hillis-Steele inclusive scan
+    const int32_t add = (int)threadIdx.x >= o ? part[threadIdx.x - o] : 0;
+    __syncthreads();
+    part[threadIdx.x] += add;
+    __syncthreads();
+  }
+  int32_t run = part[threadIdx.x] - sum;               // exclusive prefix of this chunk
+  for (int y = lo; y < hi; ++y) {
+    run += Pb[y];
+    Pb[y] = run;
+  }
+}
+
+__global__ void k_cyclic_rank(const int32_t* __restrict__ tau, const int32_t* __restrict__ P,
+                              int64_t nb, int s, int c, int32_t* __restrict__ rank) {
+  const int64_t total = nb * s * (int64_t)c;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t w = x % c, bi = x / c, i = bi % s, b = bi / s;
+    const int32_t* Pb = P + b * (int64_t)(c + 1);
+    const int64_t a = tau[b * c + i], e = a + w;
+    rank[x] = e < c ? Pb[e + 1] - Pb[a + 1] : (Pb[c] - Pb[a + 1]) + Pb[e - c + 1];
+  }
+}
+
 // ticket keys: visit (b,i,w) to column col = seq[(b*s+i)*c+w] gets key ((b*c+col)*c + w)*s + i
 __global__ void k_ticket_keys(const int32_t* __restrict__ seq, int64_t nb, int s, int c,
                               uint64_t* __restrict__ keys, uint32_t* __restrict__ vals) {
@@ -1268,6 +1316,14 @@ static mf_status build_schedule(mf_ctx* c, int32_t t) {
     }
     k_cyclic_seq<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(c->tau, c->sigma, nb, s, cc, c->seq);
     KERNEL_TRY(c);
+    int32_t* P = reinterpret_cast<int32_t*>(c->sb);       // nb (c+1) <= 2 nb c = cap: free here
+    k_tau_prefix<<<(unsigned)nb, 1024, 0, c->st>>>(c->tau, s, cc, P);
+    KERNEL_TRY(c);
+    k_cyclic_rank<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(c->tau, P, nb, s, cc, c->rank_arr);
+    KERNEL_TRY(c);
+    c->n_launch += 3;
+    c->sched_built_for = t;
+    return MF_OK;
   } else {
     k_wf_keys<<<grid_for(total, c->num_sms), 256, 0, c->st>>>(nb * s, s, cc, c->p.seed, t, c->sk0,
                                                               c->sv0);

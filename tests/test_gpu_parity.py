@@ -54,6 +54,7 @@ INDEX_CASES = [
     dict(schedule="wavefront", workers=8, wf_cols=16),
     dict(schedule="wavefront", workers=5, wf_cols=7, grid_a=4),
     dict(schedule="wavefront", workers=8, wf_cols=16, cyclic=True),
+    dict(schedule="wavefront", workers=5, wf_cols=7, grid_a=4, cyclic=True),   # closed-form ranks
 ]
 
 
