@@ -472,6 +472,13 @@ struct mf_ctx {
   uint32_t *sv0 = nullptr, *sv1 = nullptr, *sb = nullptr;
   int64_t sched_cap = 0;
   uint32_t* chunk_order = nullptr;  // Hogwild: sorted global chunk ids, blocks ascending
+  // Hogwild: the next epoch's chunk order is built on a side stream (ss) into chunk_order_alt
+  // while this epoch's SGD kernel runs (its sorts fill the SMs its retiring blocks free).
+  uint32_t* chunk_order_alt = nullptr;
+  cudaStream_t ss = nullptr;
+  cudaEvent_t ev_ss_go = nullptr, ev_ss_done = nullptr;
+  int32_t prebuilt_t = -1;           // epoch whose order chunk_order_alt holds (-1: none)
+  bool ss_pending = false;           // a side build may still use the sort scratch
   int32_t *seq = nullptr, *rank_arr = nullptr, *tickets = nullptr;
   int32_t *tau = nullptr, *sigma = nullptr;
   unsigned long long* counter = nullptr;
@@ -800,6 +807,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
 void mf_destroy(mf_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->dev);
+  if (c->ss) cudaStreamSynchronize(c->ss);
   if (c->st) cudaStreamSynchronize(c->st);
   std::vector<std::pair<void*, size_t>> all = c->sizes;
   for (auto& x : all) {
@@ -819,6 +827,9 @@ void mf_destroy(mf_ctx* c) {
     if (c->ev_free[i]) cudaEventDestroy(c->ev_free[i]);
   }
   if (c->cs) cudaStreamDestroy(c->cs);
+  for (cudaEvent_t e : {c->ev_ss_go, c->ev_ss_done})
+    if (e) cudaEventDestroy(e);
+  if (c->ss) cudaStreamDestroy(c->ss);
   if (c->own_stream && c->st) cudaStreamDestroy(c->st);
   cudaGetLastError();
   delete c;
@@ -927,6 +938,7 @@ static mf_status alloc_schedule(mf_ctx* c) {
     }
   } else {
     TRY(c->alloc(&c->chunk_order, (size_t)cap));
+    TRY(c->alloc(&c->chunk_order_alt, (size_t)cap));
   }
   return MF_OK;
 }
@@ -1268,7 +1280,17 @@ mf_status mf_load_coo(mf_ctx* c, int32_t set, int64_t nnz, const int32_t* u, con
 // ---------------------------------------------------------------------------------------------
 // per-epoch schedule (A: "Orders")
 // ---------------------------------------------------------------------------------------------
+// The main stream waits for an in-flight side-stream schedule build (they share the scratch).
+static mf_status join_side(mf_ctx* c) {
+  if (c->ss_pending) {
+    CUDA_TRY(c, cudaStreamWaitEvent(c->st, c->ev_ss_done, 0));
+    c->ss_pending = false;
+  }
+  return MF_OK;
+}
+
 static mf_status build_schedule(mf_ctx* c, int32_t t) {
+  TRY(join_side(c));
   const int64_t nb = (int64_t)c->a * c->a;
   if (c->libmf) return MF_OK;             // blocks are picked at run time from the table
   if (!c->wf) {
@@ -1560,6 +1582,29 @@ static mf_status gather_q(mf_ctx* c) {
   return MF_OK;
 }
 
+// Enqueue epoch tn's Hogwild chunk order on the side stream, into chunk_order_alt.  ev_ss_go
+// was recorded on the main stream after this epoch's schedule and before its SGD launches, so
+// the previous epoch's SGD (the last reader of chunk_order_alt) is complete when it fires.
+static mf_status prebuild_schedule(mf_ctx* c, int32_t tn) {
+  if (!c->ss) {
+    CUDA_TRY(c, cudaStreamCreateWithFlags(&c->ss, cudaStreamNonBlocking));
+    CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_ss_done, cudaEventDisableTiming));
+  }
+  CUDA_TRY(c, cudaStreamWaitEvent(c->ss, c->ev_ss_go, 0));
+  const int32_t built = c->sched_built_for;
+  std::swap(c->chunk_order, c->chunk_order_alt);
+  std::swap(c->st, c->ss);
+  const mf_status s = build_schedule(c, tn);
+  std::swap(c->st, c->ss);
+  std::swap(c->chunk_order, c->chunk_order_alt);
+  c->sched_built_for = built;
+  if (s != MF_OK) return s;
+  CUDA_TRY(c, cudaEventRecord(c->ev_ss_done, c->ss));
+  c->ss_pending = true;
+  c->prebuilt_t = tn;
+  return MF_OK;
+}
+
 mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   if (!c) return MF_E_INVAL;
   TRY(c->enter());
@@ -1572,7 +1617,19 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   c->comm_ms_acc.clear();
   CUDA_TRY(c, cudaEventRecord(c->ev_e0, c->st));
   CUDA_TRY(c, cudaEventRecord(c->ev_s0, c->st));
-  TRY(build_schedule(c, t));
+  const bool hog = !c->wf && !c->libmf && c->ch_off.back() > 0;
+  if (hog && c->prebuilt_t == t) {          // built on the side stream during the last epoch
+    TRY(join_side(c));
+    std::swap(c->chunk_order, c->chunk_order_alt);
+    c->sched_built_for = t;
+  } else {
+    TRY(build_schedule(c, t));
+  }
+  c->prebuilt_t = -1;
+  if (hog) {
+    if (!c->ev_ss_go) CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_ss_go, cudaEventDisableTiming));
+    CUDA_TRY(c, cudaEventRecord(c->ev_ss_go, c->st));
+  }
   CUDA_TRY(c, cudaEventRecord(c->ev_s1, c->st));
   if (c->libmf) {
     const int64_t nb = (int64_t)c->a * c->a;
@@ -1645,6 +1702,7 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
     }
   }
   CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
+  if (hog) TRY(prebuild_schedule(c, t + 1));   // enqueued after this epoch's SGD launches
   c->t = t + 1;
   c->have_stats = true;
   if (epoch_done) *epoch_done = c->t;
