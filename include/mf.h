@@ -91,7 +91,7 @@ typedef struct mf_params {
   int32_t grid_a;         /* strata grid a x a (0 = 1 if world == 1 else 8); a % world == 0
                              and a / world <= 16                                                */
   int32_t cyclic;         /* wavefront: 1 = cyclic column order (A: cyclic variant), needs c >= s */
-  int32_t lane_bytes;     /* Hogwild/RMSE kernel: bytes of p_u (and q_v) per lane, 16 or 32 (0 = 16).
+  int32_t lane_bytes;     /* Hogwild kernel: bytes of p_u (and q_v) per lane, 8, 16 or 32 (0 = 16).
                              Ring wavefront: 0 = default geometry (fp16/bf16 k = 128: 8 B on 32
                              lanes), 16 = 16-B lanes, 32 / 64 = half / quarter of the lanes   */
   int32_t prefetch;       /* Hogwild software-pipeline depth: samples in flight per worker, 1 or 2 (0 = 1) */

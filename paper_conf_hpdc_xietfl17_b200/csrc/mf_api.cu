@@ -717,7 +717,8 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (!(p->alpha >= 0.f) || !(p->beta >= 0.f) || !(p->lambda_p >= 0.f) || !(p->lambda_q >= 0.f))
     return MF_E_INVAL;
   if (!(p->rating_scale > 0.f) || !(p->init_scale > 0.f)) return MF_E_INVAL;
-  if (p->lane_bytes != 0 && p->lane_bytes != 16 && p->lane_bytes != 32 && p->lane_bytes != 64)
+  if (p->lane_bytes != 0 && p->lane_bytes != 8 && p->lane_bytes != 16 && p->lane_bytes != 32 &&
+      p->lane_bytes != 64)
     return MF_E_INVAL;
   if (p->prefetch < 0 || p->prefetch > 2) return MF_E_INVAL;
   if (p->wf_kernel < 0 || p->wf_kernel > 2 || p->launch_blocks < 0) return MF_E_INVAL;

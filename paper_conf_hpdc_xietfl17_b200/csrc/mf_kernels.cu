@@ -518,6 +518,7 @@ static cudaError_t hogwild_kl(const HogwildLaunch& a) {
 template <typename T, int K>
 static cudaError_t hogwild_k(const HogwildLaunch& a) {
   if (a.lane_bytes == 32) return hogwild_kl<T, K, 32>(a);
+  if (a.lane_bytes == 8) return hogwild_kl<T, K, 8>(a);
   return hogwild_kl<T, K, 16>(a);
 }
 template <typename T, int K>

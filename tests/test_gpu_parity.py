@@ -93,6 +93,7 @@ DET_CASES = [
     dict(schedule="hogwild", workers=1, grid_a=8, batch_f=64, launch_blocks=3),
     dict(schedule="hogwild", workers=1, grid_a=4, batch_f=16),
     dict(schedule="hogwild", workers=1, lane_bytes=32),
+    dict(schedule="hogwild", workers=1, lane_bytes=8),
     dict(schedule="hogwild", workers=1, prefetch=2),
 ]
 

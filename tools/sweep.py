@@ -13,7 +13,17 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 SETS = {
     "kprec": [dict(workload="netflix", k=k, storage=s) for k in (32, 64, 128, 256)
-              for s in ("fp32", "fp16")],
+              for s in ("fp32", "fp16", "bf16")],
+    # the deterministic configuration of bench.py over k and storage, and the Yahoo shape
+    "det": [dict(workload="netflix", k=k, storage=s, schedule="wavefront", workers=888,
+                 **{"wf-cols": 7680}, cyclic=True)
+            for k in (32, 64, 128, 256) for s in ("fp32", "fp16", "bf16")],
+    "yahoo2": [dict(workload="yahoo", storage="fp16"), dict(workload="yahoo", storage="fp32"),
+               dict(workload="yahoo", storage="bf16"),
+               dict(workload="yahoo", storage="fp32", schedule="wavefront", workers=888,
+                    **{"wf-cols": 15360}, cyclic=True),
+               dict(workload="yahoo", storage="fp16", schedule="wavefront", workers=888,
+                    **{"wf-cols": 15360}, cyclic=True)],
     "yahoo": [dict(workload="yahoo", storage="fp16"), dict(workload="yahoo", storage="fp32"),
               dict(workload="yahoo", storage="fp32", schedule="wavefront", workers=768),
               dict(workload="yahoo", storage="fp16", schedule="wavefront", workers=768)],
