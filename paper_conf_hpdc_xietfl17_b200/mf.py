@@ -323,6 +323,81 @@ class MF:
         return {name: getattr(s, name) for name, _ in Stats._fields_}
 
 
+# ---------------------------------------------------------------------------------------------
+# The C ABI's own names (include/mf.h), function style: each forwards to the MF method or the
+# library call above (argument marshalling only).
+# ---------------------------------------------------------------------------------------------
+def mf_abi_version() -> int:
+    return int(lib().mf_abi_version())
+
+
+def mf_status_string(status: int) -> str:
+    return lib().mf_status_string(int(status)).decode()
+
+
+def mf_params_default() -> Params:
+    p = Params()
+    lib().mf_params_default(ctypes.byref(p))
+    return p
+
+
+def mf_create(m: int, n: int, k: int = 128, **params) -> MF:
+    return MF(m, n, k, **params)
+
+
+def mf_load_coo(ctx: MF, set: str, u, v, r, on_device: bool | None = None) -> None:
+    ctx.load(u, v, r, set, on_device)
+
+
+def mf_train_epoch(ctx: MF) -> int:
+    return ctx.train_epoch()
+
+
+def mf_rmse(ctx: MF, set: str = "test") -> float:
+    return ctx.rmse(set)
+
+
+def mf_get_factors(ctx: MF, on_device: bool = False):
+    return ctx.factors(on_device)
+
+
+def mf_set_factors(ctx: MF, P=None, Q=None) -> None:
+    ctx.set_factors(P, Q)
+
+
+def mf_get_epoch(ctx: MF) -> int:
+    return ctx.epoch
+
+
+def mf_set_epoch(ctx: MF, t: int) -> None:
+    ctx.set_epoch(t)
+
+
+def mf_export_schedule(ctx: MF, what: str, epoch: int = 0) -> np.ndarray:
+    return ctx.export(what, epoch)
+
+
+def mf_get_stats(ctx: MF) -> dict:
+    return ctx.stats()
+
+
+def mf_get_launch_ms(ctx: MF) -> np.ndarray:
+    return ctx.launch_ms()
+
+
+def mf_last_error(ctx: MF) -> str:
+    msg = lib().mf_last_error(ctx.h)
+    return msg.decode() if msg else ""
+
+
+def mf_destroy(ctx: MF) -> None:
+    ctx.close()
+
+
+mf_strata_holders = strata_holders
+mf_strata_plan = strata_plan
+
+
 def _is_cuda_tensor(x) -> bool:
     try:
         import torch

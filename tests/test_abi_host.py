@@ -32,6 +32,16 @@ def test_library_exports_every_declared_symbol(L):
     assert set(names) <= set(mf.EXPORTED)
 
 
+def test_python_binding_has_every_abi_name(L):
+    """The binding is thin and named like the boundary: one same-named Python callable per
+    include/mf.h entry point (argument marshalling only)."""
+    for name in declared_symbols():
+        assert callable(getattr(mf, name, None)), name
+    assert mf.mf_abi_version() == L.mf_abi_version()
+    assert mf.mf_status_string(-6) == "MF_E_RANGE"
+    assert mf.mf_params_default().batch_f == 256
+
+
 def test_abi_version_and_status_strings(L):
     hdr = open(os.path.join(ROOT, "include", "mf.h")).read()
     assert L.mf_abi_version() == int(re.search(r"#define MF_ABI_VERSION (\d+)", hdr).group(1))

@@ -398,3 +398,21 @@ def test_adagrad_hogwild_20_epochs_matches_oracle():
         o.train_epoch()
     rg, ro = g.rmse(), o.rmse(R.ut, R.vt, R.rt)
     assert abs(rg - ro) <= 0.005 * ro, (rg, ro)
+
+
+def test_function_style_binding_matches_the_abi_call_order(tiny):
+    """create -> load_coo(train, test) -> train_epoch -> rmse / get_factors -> destroy through the
+    C ABI's own names, against the oracle (1 worker Hogwild: the serial order)."""
+    ctx = mf.mf_create(tiny.m, tiny.n, 16, schedule="hogwild", workers=1, **TABLE3_NETFLIX)
+    mf.mf_load_coo(ctx, "train", tiny.u, tiny.v, tiny.r)
+    mf.mf_load_coo(ctx, "test", tiny.ut, tiny.vt, tiny.rt)
+    assert mf.mf_train_epoch(ctx) == 1 and mf.mf_get_epoch(ctx) == 1
+    rg = mf.mf_rmse(ctx, "test")
+    Pg, Qg = mf.mf_get_factors(ctx)
+    assert mf.mf_get_stats(ctx)["updates"] == tiny.N and mf.mf_last_error(ctx) == ""
+    mf.mf_destroy(ctx)
+    o = po.Oracle(tiny.m, tiny.n, 16, tiny.u, tiny.v, tiny.r, schedule="hogwild", **TABLE3_NETFLIX)
+    o.train_epoch()
+    Po, Qo = o.factors()
+    assert np.abs(Pg - Po).max() <= 1e-4 and np.abs(Qg - Qo).max() <= 1e-4
+    assert abs(rg - o.rmse(tiny.ut, tiny.vt, tiny.rt)) <= 1e-5 * rg
