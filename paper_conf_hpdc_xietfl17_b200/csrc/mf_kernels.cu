@@ -29,8 +29,15 @@ constexpr bool narrow16_ring(int K, int S) { return K * S == 64; }
 // f consecutive slots of its chunk serially.  Persistent grid: workers loop until the list is
 // exhausted.  The chunk list of a launch is the concatenation of up to kMaxSegs block segments.
 // ---------------------------------------------------------------------------------------------
+// 5 resident blocks (40 warps) per SM: 48 registers, a few bytes of stack.  Yahoo-shaped
+// (DRAM-bound) 34.9 -> 33.8 ms/epoch against 4 blocks at 64 registers, Netflix unchanged (hot
+// rows); the ADAGRAD, depth-2 and 32-B-per-lane variants keep the compiler's choice.
+#ifndef MF_HOG_MINB
+#define MF_HOG_MINB 5
+#endif
 template <typename T, int K, int L, int D, bool ADA>
-__global__ void __launch_bounds__(256) k_hogwild(const Rating* __restrict__ slots,
+__global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L > 16) ? 1 : MF_HOG_MINB)
+    k_hogwild(const Rating* __restrict__ slots,
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
                                                  unsigned long long* __restrict__ counter,
                                                  int workers, T* __restrict__ P, T* __restrict__ Q,
