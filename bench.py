@@ -250,7 +250,11 @@ def main():
     kw = dict(schedule=args.schedule, storage=args.storage, workers=args.workers,
               wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes, prefetch=args.prefetch,
               wf_kernel=args.wf_kernel, staged=args.staged, grid_a=args.grid_a,
-              batch_f=args.batch_f or 256,
+              # N > 1: f = 64.  Each rank's sub-epoch launch holds ~1/64 of the ratings, so
+              # 256-sample chunks leave ~1.6 chunks per worker and a quantised tail; emulated on
+              # Yahoo at G = 8: 49.3 (f = 256) -> 54.3 G updates/s (f = 64), same RMSE
+              # (profiles/r01_scaling_hot_rows.md section 6; f is Eq. 8's free batch)
+              batch_f=args.batch_f or (64 if world > 1 else 256),
               lr_rule=args.lr_rule, seed=42,
               device=local, rank=rank, world=world, nccl_id=nccl_id, **hp)
     torch.cuda.synchronize()
