@@ -222,7 +222,7 @@ def config_of(args, R):
     return {"workload": f"{args.workload}-shaped synthetic (Table 2 shape, power-law skew)",
             "m": R.m, "n": R.n, "N_train": R.N, "N_test": R.Ntest, "k": args.k,
             "storage": args.storage, "schedule": args.schedule,
-            "batch_f": args.batch_f or 256,
+            "batch_f": args.batch_f or (64 if args.gpus > 1 else 256),
             "parallelism": f"dsgd-strata{args.gpus}" if args.gpus > 1 else "1gpu",
             "staged": bool(args.staged), "grid_a": args.grid_a or (8 if args.gpus > 1 else 1),
             "l2": "inputs larger than L2 (COO %.2f GB per epoch); model P+Q stays cached as in "
