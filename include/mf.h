@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define MF_ABI_VERSION 2
+#define MF_ABI_VERSION 3
 
 typedef struct mf_ctx mf_ctx; /* opaque, owned by the library */
 
@@ -192,6 +192,9 @@ typedef struct mf_stats {
   int64_t updates;          /* samples updated by this rank in the epoch */
   int64_t bytes_per_update; /* algorithmic: 12 + 4*k*sizeof(storage) (north_star; Eq. 5)  */
   int32_t workers, lanes, grid, block;
+  int64_t h2d_bytes;        /* staged mode: bytes copied host -> device for the epoch's ratings
+                               (10 per rating when n <= 65535: packed u, v16, r; else 12; +2
+                               with the wavefront's duplicate distances)                      */
 } mf_stats;
 mf_status mf_get_stats(mf_ctx* ctx, mf_stats* out);
 

@@ -203,6 +203,31 @@ __global__ void k_dupdist(const Rating* __restrict__ slots, int64_t N, Grid G, i
   }
 }
 
+// Packed staging: 12-B slots <-> (u int32, v uint16, r fp32).  Sentinel pad slots (u = v = -1)
+// keep u = -1 and get v back from it; real v < n <= 65535.
+__global__ void k_split_slots(const Rating* __restrict__ s, int64_t N, int32_t* __restrict__ u,
+                              uint16_t* __restrict__ v, float* __restrict__ r) {
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < N;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const Rating a = s[x];
+    u[x] = a.u;
+    v[x] = (uint16_t)a.v;
+    r[x] = a.r;
+  }
+}
+__global__ void k_expand_slots(const int32_t* __restrict__ u, const uint16_t* __restrict__ v,
+                               const float* __restrict__ r, int64_t N, Rating* __restrict__ s) {
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < N;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t uu = __ldcs(u + x);
+    Rating a;
+    a.u = uu;
+    a.v = uu < 0 ? -1 : (int32_t)__ldcs(v + x);
+    a.r = __ldcs(r + x);
+    s[x] = a;
+  }
+}
+
 // Alg. 1 l.3 (R5): X[rho[id]][d] = round_S((float)U24(S, id*k+d) * 2^-24 * amp),
 // keyed by the ORIGINAL id (A: S_P / S_Q).
 template <typename T>
@@ -510,6 +535,17 @@ struct mf_ctx {
   int *lm_lock = nullptr, *lm_row = nullptr, *lm_col = nullptr, *lm_done = nullptr, *lm_rem = nullptr;
 
   bool staged = false;
+  // Packed staging (n <= 65535): the pinned host copy and the H2D stream carry 10 B per rating
+  // (u int32, v uint16, r fp32, structure of arrays) instead of the 12-B slot; the compute
+  // stream expands each staged stratum back into 12-B slots before its SGD launch.
+  bool stg_packed = false;
+  int32_t* h_u = nullptr;
+  uint16_t* h_v16 = nullptr;
+  float* h_r = nullptr;
+  int32_t* stg_u[2] = {nullptr, nullptr};
+  uint16_t* stg_v16[2] = {nullptr, nullptr};
+  float* stg_r[2] = {nullptr, nullptr};
+  int64_t stg_len[2] = {0, 0};
   Rating* h_slots = nullptr;
   uint16_t* h_dup = nullptr;
   Rating* stg[2] = {nullptr, nullptr};
@@ -822,6 +858,9 @@ void mf_destroy(mf_ctx* c) {
   if (c->comm) mf::Comm::destroy(c->comm);
   if (c->cs) cudaStreamSynchronize(c->cs);
   if (c->h_slots) cudaFreeHost(c->h_slots);
+  if (c->h_u) cudaFreeHost(c->h_u);
+  if (c->h_v16) cudaFreeHost(c->h_v16);
+  if (c->h_r) cudaFreeHost(c->h_r);
   if (c->h_dup) cudaFreeHost(c->h_dup);
   for (int i = 0; i < 2; ++i) {
     if (c->ev_h2d[i]) cudaEventDestroy(c->ev_h2d[i]);
@@ -950,8 +989,32 @@ static mf_status alloc_schedule(mf_ctx* c) {
 static mf_status setup_staging(mf_ctx* c) {
   CUDA_TRY(c, cudaStreamSynchronize(c->st));
   const size_t ns = (size_t)std::max<int64_t>(c->nslots, 1);
-  CUDA_TRY(c, cudaMallocHost(&c->h_slots, ns * sizeof(Rating)));
-  CUDA_TRY(c, cudaMemcpyAsync(c->h_slots, c->slots, ns * sizeof(Rating), cudaMemcpyDeviceToHost, c->st));
+  c->stg_packed = c->n <= 65535;
+  if (c->stg_packed) {
+    int32_t* du = nullptr;
+    uint16_t* dv = nullptr;
+    float* dr = nullptr;
+    TRY(c->alloc(&du, ns));
+    TRY(c->alloc(&dv, ns));
+    TRY(c->alloc(&dr, ns));
+    if (c->nslots > 0) {
+      k_split_slots<<<grid_for(c->nslots, c->num_sms), 256, 0, c->st>>>(c->slots, c->nslots, du, dv, dr);
+      KERNEL_TRY(c);
+    }
+    CUDA_TRY(c, cudaMallocHost(&c->h_u, ns * 4));
+    CUDA_TRY(c, cudaMallocHost(&c->h_v16, ns * 2));
+    CUDA_TRY(c, cudaMallocHost(&c->h_r, ns * 4));
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_u, du, ns * 4, cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_v16, dv, ns * 2, cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_r, dr, ns * 4, cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    c->release(du);
+    c->release(dv);
+    c->release(dr);
+  } else {
+    CUDA_TRY(c, cudaMallocHost(&c->h_slots, ns * sizeof(Rating)));
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_slots, c->slots, ns * sizeof(Rating), cudaMemcpyDeviceToHost, c->st));
+  }
   if (c->dup) {
     CUDA_TRY(c, cudaMallocHost(&c->h_dup, ns * sizeof(uint16_t)));
     CUDA_TRY(c, cudaMemcpyAsync(c->h_dup, c->dup, ns * sizeof(uint16_t), cudaMemcpyDeviceToHost, c->st));
@@ -976,6 +1039,11 @@ static mf_status setup_staging(mf_ctx* c) {
   for (int i = 0; i < 2; ++i) {
     TRY(c->alloc(&c->stg[i], (size_t)cap));
     if (c->h_dup) TRY(c->alloc(&c->stg_dup[i], (size_t)cap));
+    if (c->stg_packed) {
+      TRY(c->alloc(&c->stg_u[i], (size_t)cap));
+      TRY(c->alloc(&c->stg_v16[i], (size_t)cap));
+      TRY(c->alloc(&c->stg_r[i], (size_t)cap));
+    }
     CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_h2d[i], cudaEventDisableTiming));
     CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_free[i], cudaEventDisableTiming));
     CUDA_TRY(c, cudaEventRecord(c->ev_free[i], c->st));
@@ -1003,14 +1071,24 @@ static mf_status stage(mf_ctx* c, int32_t t, int32_t j, int buf) {
     const int64_t lo = c->blk_off[(size_t)b], len = c->blk_off[(size_t)b + 1] - lo;
     c->stg_shift[buf].push_back({b, off - lo});
     if (len == 0) continue;
-    CUDA_TRY(c, cudaMemcpyAsync(c->stg[buf] + off, c->h_slots + lo, (size_t)len * sizeof(Rating),
-                                cudaMemcpyHostToDevice, c->cs));
+    if (c->stg_packed) {
+      CUDA_TRY(c, cudaMemcpyAsync(c->stg_u[buf] + off, c->h_u + lo, (size_t)len * 4,
+                                  cudaMemcpyHostToDevice, c->cs));
+      CUDA_TRY(c, cudaMemcpyAsync(c->stg_v16[buf] + off, c->h_v16 + lo, (size_t)len * 2,
+                                  cudaMemcpyHostToDevice, c->cs));
+      CUDA_TRY(c, cudaMemcpyAsync(c->stg_r[buf] + off, c->h_r + lo, (size_t)len * 4,
+                                  cudaMemcpyHostToDevice, c->cs));
+    } else {
+      CUDA_TRY(c, cudaMemcpyAsync(c->stg[buf] + off, c->h_slots + lo, (size_t)len * sizeof(Rating),
+                                  cudaMemcpyHostToDevice, c->cs));
+    }
     if (c->h_dup)
       CUDA_TRY(c, cudaMemcpyAsync(c->stg_dup[buf] + off, c->h_dup + lo, (size_t)len * 2,
                                   cudaMemcpyHostToDevice, c->cs));
-    c->h2d_bytes += len * (int64_t)(sizeof(Rating) + (c->h_dup ? 2 : 0));
+    c->h2d_bytes += len * (int64_t)((c->stg_packed ? 10 : sizeof(Rating)) + (c->h_dup ? 2 : 0));
     off += len;
   }
+  c->stg_len[buf] = off;
   CUDA_TRY(c, cudaEventRecord(c->ev_h2d[buf], c->cs));
   c->staged_t = t;
   c->staged_j = j;
@@ -1615,6 +1693,7 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   c->n_sgd = 0;
   c->n_launch = 0;
   c->updates = 0;
+  c->h2d_bytes = 0;
   c->comm_ms_acc.clear();
   CUDA_TRY(c, cudaEventRecord(c->ev_e0, c->st));
   CUDA_TRY(c, cudaEventRecord(c->ev_s0, c->st));
@@ -1691,6 +1770,17 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
       const bool last = j + 1 == c->a;
       TRY(stage(c, last ? t + 1 : t, last ? 0 : j + 1, 1 - buf));   // overlap the next copy
       CUDA_TRY(c, cudaStreamWaitEvent(c->st, c->ev_h2d[buf], 0));
+      if (c->stg_packed) {
+        if (c->stg_len[buf] > 0) {
+          k_expand_slots<<<grid_for(c->stg_len[buf], c->num_sms), 256, 0, c->st>>>(
+              c->stg_u[buf], c->stg_v16[buf], c->stg_r[buf], c->stg_len[buf], c->stg[buf]);
+          KERNEL_TRY(c);
+          ++c->n_launch;
+        }
+        // the packed buffers are free again once expanded (the slots are stream-ordered);
+        // not so the wavefront's duplicate distances, which the SGD launch reads in place
+        if (!c->h_dup) CUDA_TRY(c, cudaEventRecord(c->ev_free[buf], c->st));
+      }
     }
     const int per_launch = (!c->wf && c->p.launch_blocks > 0) ? c->p.launch_blocks : std::max(nb, 1);
     for (int b0 = 0; b0 < nb; b0 += per_launch)
@@ -1698,7 +1788,7 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
                                               blocks.begin() + std::min(nb, b0 + per_launch)),
                       g, buf));
     if (c->staged) {
-      CUDA_TRY(c, cudaEventRecord(c->ev_free[buf], c->st));
+      if (!c->stg_packed || c->h_dup) CUDA_TRY(c, cudaEventRecord(c->ev_free[buf], c->st));
       c->cur_buf = 1 - buf;
     }
   }
@@ -1752,6 +1842,7 @@ mf_status mf_get_stats(mf_ctx* c, mf_stats* out) {
   out->launches = c->n_launch;
   out->updates = c->updates;
   out->bytes_per_update = 12 + 4 * (int64_t)c->k * c->ssize() + (c->GP ? 16 * (int64_t)c->k : 0);
+  out->h2d_bytes = c->h2d_bytes;
   out->workers = c->last_workers;
   out->lanes = c->last_lanes;
   out->grid = c->last_grid;

@@ -63,7 +63,7 @@ class Stats(ctypes.Structure):
                 ("sgd_launches", ctypes.c_int64), ("launches", ctypes.c_int64),
                 ("updates", ctypes.c_int64), ("bytes_per_update", ctypes.c_int64),
                 ("workers", ctypes.c_int32), ("lanes", ctypes.c_int32),
-                ("grid", ctypes.c_int32), ("block", ctypes.c_int32)]
+                ("grid", ctypes.c_int32), ("block", ctypes.c_int32), ("h2d_bytes", ctypes.c_int64)]
 
 
 _lib = None

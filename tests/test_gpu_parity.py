@@ -313,14 +313,18 @@ def test_checkpoint_resume_equals_uninterrupted(tiny):
 @pytest.mark.parametrize("kw", [dict(schedule="wavefront", workers=4, wf_cols=5, grid_a=8),
                                 dict(schedule="wavefront", workers=4, wf_cols=5, grid_a=1),
                                 dict(schedule="hogwild", workers=1, grid_a=8, batch_f=64),
-                                dict(schedule="wavefront", workers=6, wf_cols=9, grid_a=4, k=128)])
+                                dict(schedule="wavefront", workers=6, wf_cols=9, grid_a=4, k=128),
+                                dict(schedule="hogwild", workers=1, grid_a=4, batch_f=64, wide=True),
+                                dict(schedule="wavefront", workers=4, wf_cols=5, grid_a=2, wide=True)])
 def test_staged_equals_resident(kw):
     """Section 6.2 out-of-core mode: ratings in pinned host memory, streamed per stratum through
     two HBM buffers (copy stream overlapping compute, also across epochs).  Same order, so the
-    deterministic result is bit-identical to the resident run."""
+    deterministic result is bit-identical to the resident run.  n <= 65535 stages packed 10-B
+    records (expanded on the GPU); `wide` (n = 70,000) stages the 12-B slots as they are."""
     kw = dict(kw)
     k = kw.pop("k", 32)
-    R = ragged()
+    R = ragged() if not kw.pop("wide", False) else synth.uniform(
+        m=331, n=70_000, N=12_345, seed=7, mu=0.5, rank=3, noise=0.1, Ntest=777)
     out = []
     for staged in (False, True):
         g = mf.MF(R.m, R.n, k, staged=staged, **TABLE3_NETFLIX, **kw)
@@ -328,6 +332,11 @@ def test_staged_equals_resident(kw):
         g.load(R.ut, R.vt, R.rt, "test")
         for _ in range(3):
             g.train_epoch()
+        if staged:
+            per = 10 if R.n <= 65535 else 12
+            per += 2 if kw["schedule"] == "wavefront" else 0
+            h2d = g.stats()["h2d_bytes"]      # ~ one epoch: its later strata + the next epoch's first
+            assert h2d % per == 0 and 0.5 * R.N <= h2d / per <= 1.5 * R.N, (h2d, per)
         out.append((g.factors(), g.rmse()))
         g.close()
     (P0, Q0), r0 = out[0]
