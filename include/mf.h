@@ -104,6 +104,8 @@ typedef struct mf_params {
                              preprocessing the bucketed ratings live in pinned host memory and
                              each stratum's blocks stream into one of two HBM buffers on a copy
                              stream while the previous stratum computes; P, Q stay resident.
+                             When n <= 65535 the host copy and the H2D stream carry 10-B
+                             records (u int32, v uint16, r fp32) expanded on the GPU.
                              Same order and result as resident.  0 = ratings resident in HBM */
   int32_t wf_kernel;      /* wavefront kernel: 0 = auto = 1 = ring-staged (cp.async smem ring),
                              2 = register pipeline; both give the same result                   */
