@@ -340,8 +340,10 @@ def run_deterministic(args, R, hp, stream):
     line."""
     from paper_conf_hpdc_xietfl17_b200 import mf
     steps, warm = max(3, args.steps // 2), 2
-    m = mf.MF(R.m, R.n, args.k, stream=stream, schedule="wavefront", storage="fp32", workers=888,
-              wf_cols=7680, cyclic=True, seed=42, **hp)
+    s_w = min(888, max(1, R.m // 4))                  # (clamped only for --fraction test runs)
+    c_w = max(s_w, min(7680, R.n))
+    m = mf.MF(R.m, R.n, args.k, stream=stream, schedule="wavefront", storage="fp32", workers=s_w,
+              wf_cols=c_w, cyclic=True, seed=42, **hp)
     m.load(R.u, R.v, R.r, "train")
     m.load(R.ut, R.vt, R.rt, "test")
     for _ in range(warm):
@@ -362,7 +364,7 @@ def run_deterministic(args, R, hp, stream):
     hbm, _ = peaks()
     bpu = st["bytes_per_update"]
     achieved = upd * bpu / (float(np.sum(sgd)) / 1000.0) / 1e9
-    out = {"schedule": "wavefront (deterministic, cyclic, s=888, c=7680)", "storage": "fp32",
+    out = {"schedule": f"wavefront (deterministic, cyclic, s={s_w}, c={c_w})", "storage": "fp32",
            "value": upd / (ms / 1000.0), "unit": "updates/s", "ms_per_step": ms / steps,
            "steps": steps, "warmup": warm, "test_rmse": m.rmse("test"),
            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
