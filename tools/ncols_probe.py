@@ -25,6 +25,7 @@ ap.add_argument("--storage", default="fp16")
 ap.add_argument("--workers", default="0")
 ap.add_argument("--mu", type=float, default=0.0)
 ap.add_argument("--epochs", type=int, default=4)
+ap.add_argument("--k", type=int, default=128)
 args = ap.parse_args()
 
 for n in [int(x) for x in args.ns.split(",")]:
@@ -34,7 +35,7 @@ for n in [int(x) for x in args.ns.split(",")]:
         dv = torch.bincount(R.v.long(), minlength=n)
         top = float(dv.max()) / R.N
         for w in [int(x) for x in args.workers.split(",")]:
-            g = mf.MF(R.m, R.n, 128, storage=args.storage, workers=w, lambda_p=0.03, alpha=0.08,
+            g = mf.MF(R.m, R.n, args.k, storage=args.storage, workers=w, lambda_p=0.03, alpha=0.08,
                       beta=0.3, seed=42)
             g.load(R.u, R.v, R.r)
             g.load(R.ut, R.vt, R.rt, "test")
