@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define MF_ABI_VERSION 3
+#define MF_ABI_VERSION 4
 
 typedef struct mf_ctx mf_ctx; /* opaque, owned by the library */
 
@@ -191,7 +191,9 @@ mf_status mf_export_schedule(mf_ctx* ctx, int32_t what, int32_t epoch, int64_t* 
 typedef struct mf_stats {
   double epoch_ms, sgd_ms, sched_ms, comm_ms;
   int64_t sgd_launches, launches;
-  int64_t updates;          /* samples updated by this rank in the epoch */
+  int64_t updates;          /* samples updated by this rank in the epoch, counted ON THE DEVICE
+                               by the SGD kernels (non-sentinel samples each worker ran; Eq. 7,
+                               P:L253: an epoch is N updates)                                  */
   int64_t bytes_per_update; /* algorithmic: 12 + 4*k*sizeof(storage) (north_star; Eq. 5)  */
   int32_t workers, lanes, grid, block;
   int64_t h2d_bytes;        /* staged mode: bytes copied host -> device for the epoch's ratings
@@ -199,6 +201,17 @@ typedef struct mf_stats {
                                with the wavefront's duplicate distances)                      */
 } mf_stats;
 mf_status mf_get_stats(mf_ctx* ctx, mf_stats* out);
+
+/* Exactly-once evidence (Eq. 7; SURVEY 8(c) "each sample exactly once per epoch").
+ * Every SGD kernel records, on the device, one claim per work unit it runs: a Hogwild chunk of
+ * f consecutive slots, a wavefront sub-block, a LIBMF block.  Units are disjoint slot ranges
+ * and a worker runs every slot of the unit it claimed, so "every unit claimed exactly once per
+ * epoch" plus mf_stats.updates == N (the kernels' own count of non-sentinel samples) means
+ * every sample was updated exactly once.  This call compares each unit's claim count since
+ * mf_load_coo with the number of epochs run since then (0 for wavefront sub-blocks of blocks
+ * this rank does not train) and writes the number of mismatching units to *bad_units, the
+ * number of units to *units and the epochs to *epochs (either may be NULL).  Synchronises. */
+mf_status mf_check_visits(mf_ctx* ctx, int64_t* bad_units, int64_t* units, int32_t* epochs);
 
 /* Per-launch device times (ms, CUDA events) of the SGD launches of the last epoch, in launch
  * order (synchronises).  With ms == NULL only *n is set; otherwise *n must be >= the count and

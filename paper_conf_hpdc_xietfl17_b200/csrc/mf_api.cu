@@ -507,6 +507,14 @@ struct mf_ctx {
   int32_t *seq = nullptr, *rank_arr = nullptr, *tickets = nullptr;
   int32_t *tau = nullptr, *sigma = nullptr;
   unsigned long long* counter = nullptr;
+  // Exactly-once evidence (Eq. 7): per work unit (Hogwild chunk / wavefront sub-block /
+  // LIBMF block) the number of claims since load, and the device count of the samples the SGD
+  // kernels updated in the current epoch.  mf_check_visits compares the former with epochs_run.
+  unsigned* visits = nullptr;
+  int64_t n_units = 0;
+  unsigned long long* upd_dev = nullptr;
+  unsigned long long* chk_dev = nullptr;
+  int32_t epochs_run = 0;
   double* rm_partial = nullptr;
   double* rm_out = nullptr;
   void* tmp = nullptr;
@@ -518,7 +526,6 @@ struct mf_ctx {
   cudaEvent_t ev_e0 = nullptr, ev_e1 = nullptr, ev_s0 = nullptr, ev_s1 = nullptr;
   cudaEvent_t ev_c0 = nullptr, ev_c1 = nullptr;
   int n_sgd = 0, n_launch = 0;
-  int64_t updates = 0;
   int last_workers = 0, last_lanes = 0, last_grid = 0, last_block = 0;
   bool have_stats = false;
   std::vector<double> comm_ms_acc;
@@ -636,6 +643,38 @@ struct mf_ctx {
     e = cub::DeviceRadixSort::SortPairs(tmp, bytes, kin, kout, vin, vout, n_items, 0, end_bit, st);
     if (e != cudaSuccess) return cuda_fail(e, "cub sort", __LINE__);
     return MF_OK;
+  }
+  // Error path of mf_load_coo: release every device allocation made since `before` (a snapshot
+  // of `sizes` taken on entry) and null the members that pointed at them, so the ctx stays
+  // usable and a retried load does not accumulate the failed attempt's buffers.
+  void drop_allocations_since(const std::vector<std::pair<void*, size_t>>& before) {
+    std::vector<void*> fresh;
+    for (auto& x : sizes) {
+      bool old = false;
+      for (auto& y : before) old = old || y.first == x.first;
+      if (!old) fresh.push_back(x.first);
+    }
+    void** members[] = {
+        (void**)&slots, (void**)&slot_pos, (void**)&perm, (void**)&rho_r, (void**)&rho_c, &P, &Q,
+        (void**)&test, (void**)&dup, (void**)&sub_off, (void**)&d_choff, (void**)&sk0,
+        (void**)&sk1, (void**)&sv0, (void**)&sv1, (void**)&sb, (void**)&chunk_order,
+        (void**)&chunk_order_alt, (void**)&seq, (void**)&rank_arr, (void**)&tickets,
+        (void**)&tau, (void**)&sigma, &tmp, (void**)&GP, (void**)&GQ, (void**)&d_blk_off,
+        (void**)&d_blk_len, (void**)&lm_lock, (void**)&lm_row, (void**)&lm_col, (void**)&lm_done,
+        (void**)&lm_rem, (void**)&stg[0], (void**)&stg[1], (void**)&stg_dup[0],
+        (void**)&stg_dup[1], (void**)&stg_u[0], (void**)&stg_u[1], (void**)&stg_v16[0],
+        (void**)&stg_v16[1], (void**)&stg_r[0], (void**)&stg_r[1], (void**)&visits};
+    for (void* ptr : fresh) {
+      for (void** m : members)
+        if (*m == ptr) *m = nullptr;
+      void* q = ptr;
+      release(q);
+      if (ptr == tmp) tmp = nullptr;
+    }
+    if (!tmp) tmp_bytes = 0;
+    for (void** h : {(void**)&h_slots, (void**)&h_u, (void**)&h_v16, (void**)&h_r, (void**)&h_dup})
+      if (*h) { cudaFreeHost(*h); *h = nullptr; }
+    cudaGetLastError();
   }
   int ssize() const { return p.storage == MF_FP32 ? 4 : 2; }
   int lo_row_seg() const { return rank * (a / G); }
@@ -833,7 +872,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
     }
   }
   if (c->alloc(&c->counter, 1) || c->alloc(&c->rm_partial, (size_t)c->num_sms * 4) ||
-      c->alloc(&c->rm_out, 2)) {
+      c->alloc(&c->rm_out, 2) || c->alloc(&c->upd_dev, 1) || c->alloc(&c->chk_dev, 1)) {
     mf_destroy(c);
     return MF_E_NOMEM;
   }
@@ -844,7 +883,11 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
 void mf_destroy(mf_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->dev);
+  // every stream that may still touch ctx memory drains before the stream-ordered frees: the
+  // side schedule stream, the staging copy stream (an epoch ends by queueing the next
+  // stratum's H2D into a staging buffer on cs, which nothing on st waits for) and st itself
   if (c->ss) cudaStreamSynchronize(c->ss);
+  if (c->cs) cudaStreamSynchronize(c->cs);
   if (c->st) cudaStreamSynchronize(c->st);
   std::vector<std::pair<void*, size_t>> all = c->sizes;
   for (auto& x : all) {
@@ -856,7 +899,6 @@ void mf_destroy(mf_ctx* c) {
   for (cudaEvent_t e : {c->ev_e0, c->ev_e1, c->ev_s0, c->ev_s1, c->ev_c0, c->ev_c1})
     if (e) cudaEventDestroy(e);
   if (c->comm) mf::Comm::destroy(c->comm);
-  if (c->cs) cudaStreamSynchronize(c->cs);
   if (c->h_slots) cudaFreeHost(c->h_slots);
   if (c->h_u) cudaFreeHost(c->h_u);
   if (c->h_v16) cudaFreeHost(c->h_v16);
@@ -1288,14 +1330,23 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
     CUDA_TRY(c, cudaMemsetAsync(c->GQ, 0, (size_t)(c->n * c->k) * 4, c->st));
   }
   TRY(alloc_schedule(c));
+  c->n_units = c->libmf ? nb : (c->wf ? nbuckets : c->ch_off.back());
+  TRY(c->alloc(&c->visits, (size_t)std::max<int64_t>(c->n_units, 1)));
+  CUDA_TRY(c, cudaMemsetAsync(c->visits, 0, (size_t)std::max<int64_t>(c->n_units, 1) * 4, c->st));
+  c->epochs_run = 0;
   if (c->staged) TRY(setup_staging(c));
   CUDA_TRY(c, cudaStreamSynchronize(c->st));
   c->train_loaded = true;
   return MF_OK;
 }
 
+static mf_status join_side(mf_ctx* c);
+
 static mf_status load_test(mf_ctx* c, int64_t N, const int32_t* u, const int32_t* v, const float* r,
                            int on_device) {
+  // the side stream may still be building the next epoch's chunk order in the shared sort
+  // scratch (tmp), which the world > 1 test-set selection below reuses
+  TRY(join_side(c));
   const int32_t *du, *dv;
   const float* dr;
   int32_t *ou, *ov;
@@ -1344,16 +1395,24 @@ mf_status mf_load_coo(mf_ctx* c, int32_t set, int64_t nnz, const int32_t* u, con
   if (!c) return MF_E_INVAL;
   TRY(c->enter());
   if (nnz < 0 || (nnz > 0 && (!u || !v || !r))) return c->fail(MF_E_INVAL, "bad COO arguments");
+  const std::vector<std::pair<void*, size_t>> before = c->sizes;
+  mf_status s = MF_OK;
   if (set == MF_TRAIN) {
     if (c->train_loaded) return c->fail(MF_E_STATE, "train set already loaded");
-    return load_train(c, nnz, u, v, r, on_device);
-  }
-  if (set == MF_TEST) {
+    s = load_train(c, nnz, u, v, r, on_device);
+  } else if (set == MF_TEST) {
     if (!c->train_loaded) return c->fail(MF_E_STATE, "load the train set first");
     if (c->test_loaded) return c->fail(MF_E_STATE, "test set already loaded");
-    return load_test(c, nnz, u, v, r, on_device);
+    s = load_test(c, nnz, u, v, r, on_device);
+  } else {
+    return c->fail(MF_E_INVAL, "set must be MF_TRAIN or MF_TEST");
   }
-  return c->fail(MF_E_INVAL, "set must be MF_TRAIN or MF_TEST");
+  if (s != MF_OK && c->sticky == MF_OK) {
+    // recoverable failure (MF_E_RANGE, MF_E_NOMEM, ...): the ctx stays usable
+    cudaStreamSynchronize(c->st);
+    c->drop_allocations_since(before);
+  }
+  return s;
 }
 
 // ---------------------------------------------------------------------------------------------
@@ -1521,7 +1580,6 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
       segs.begin[segs.n] = c->ch_off[(size_t)b];
       segs.prefix[segs.n + 1] = segs.prefix[segs.n] + nch;
       segs.shift[segs.n] = slot_shift(c, buf, b);
-      c->updates += c->blk_len[(size_t)b];
       ++segs.n;
     }
     if (segs.n == 0) return MF_OK;
@@ -1536,6 +1594,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     L.ada = ada_args(c);
     if (L.ada.GP) L.g = c->p.alpha;        // ADAGRAD: constant alpha, no Eq. 9 decay
     L.out_workers = &c->last_workers; L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
+    L.visits = c->visits; L.upd = c->upd_dev;
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
     CUDA_TRY(c, launch_hogwild(L));
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd + 1), c->st));
@@ -1560,6 +1619,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     L.ada = ada_args(c);
     if (L.ada.GP) L.g = c->p.alpha;
     L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
+    L.visits = c->visits + base; L.upd = c->upd_dev;
     // Diagnostics only (MF_PROFILE_WAVES=1): per-worker clock64 totals of ticket waits and
     // sub-block runs, summarised on stderr after the launch (synchronises).
     static const bool kProfWaves = std::getenv("MF_PROFILE_WAVES") != nullptr;
@@ -1607,7 +1667,6 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd + 1), c->st));
     c->last_workers = c->s;
     c->last_block = 128;
-    c->updates += c->blk_len[(size_t)b];
     ++c->n_sgd;
     ++c->n_launch;
   }
@@ -1692,9 +1751,9 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   const float g = gamma_of(c->p.alpha, c->p.beta, t);   // Eq. 9
   c->n_sgd = 0;
   c->n_launch = 0;
-  c->updates = 0;
   c->h2d_bytes = 0;
   c->comm_ms_acc.clear();
+  CUDA_TRY(c, cudaMemsetAsync(c->upd_dev, 0, sizeof(unsigned long long), c->st));
   CUDA_TRY(c, cudaEventRecord(c->ev_e0, c->st));
   CUDA_TRY(c, cudaEventRecord(c->ev_s0, c->st));
   const bool hog = !c->wf && !c->libmf && c->ch_off.back() > 0;
@@ -1726,18 +1785,19 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
     L.workers = c->p.workers > 0 ? c->p.workers : std::max(1, c->a / 2);
     L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q;
     L.seed = make_stream(c->p.seed, 11, (uint64_t)t, 0); L.stream = c->st; L.out_lanes = &c->last_lanes;
+    L.visits = c->visits; L.upd = c->upd_dev;
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 0), c->st));
     CUDA_TRY(c, launch_libmf(L));
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 1), c->st));
     CUDA_TRY(c, cudaStreamSynchronize(c->st));   // the host-side copy of `rem` must outlive it
     c->n_sgd = 1;
     c->n_launch += 1;
-    c->updates = c->N;
     c->last_workers = L.workers;
     c->last_grid = L.workers;
     c->last_block = 32;
     CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
     c->t = t + 1;
+    ++c->epochs_run;
     c->have_stats = true;
     if (epoch_done) *epoch_done = c->t;
     return MF_OK;
@@ -1795,6 +1855,7 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
   if (hog) TRY(prebuild_schedule(c, t + 1));   // enqueued after this epoch's SGD launches
   c->t = t + 1;
+  ++c->epochs_run;
   c->have_stats = true;
   if (epoch_done) *epoch_done = c->t;
   return MF_OK;
@@ -1840,13 +1901,41 @@ mf_status mf_get_stats(mf_ctx* c, mf_stats* out) {
   out->comm_ms = std::max(0.0, out->epoch_ms - out->sched_ms - sgd);
   out->sgd_launches = c->n_sgd;
   out->launches = c->n_launch;
-  out->updates = c->updates;
+  unsigned long long upd = 0;     // counted by the SGD kernels themselves (non-sentinel samples)
+  CUDA_TRY(c, cudaMemcpyAsync(&upd, c->upd_dev, 8, cudaMemcpyDeviceToHost, c->st));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  out->updates = (int64_t)upd;
   out->bytes_per_update = 12 + 4 * (int64_t)c->k * c->ssize() + (c->GP ? 16 * (int64_t)c->k : 0);
   out->h2d_bytes = c->h2d_bytes;
   out->workers = c->last_workers;
   out->lanes = c->last_lanes;
   out->grid = c->last_grid;
   out->block = c->last_block;
+  return MF_OK;
+}
+
+mf_status mf_check_visits(mf_ctx* c, int64_t* bad_units, int64_t* units, int32_t* epochs) {
+  if (!c || !bad_units) return MF_E_INVAL;
+  TRY(c->enter());
+  if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
+  CUDA_TRY(c, cudaMemsetAsync(c->chk_dev, 0, 8, c->st));
+  const unsigned e = (unsigned)c->epochs_run;
+  if (c->wf) {
+    // a strata block's s*c sub-blocks are visited once per epoch when the rank trains the block
+    // (it owns the row segment and the block holds ratings); the others never
+    const int64_t per = (int64_t)c->s * c->c, nb = (int64_t)c->a * c->a;
+    for (int64_t b = 0; b < nb; ++b)
+      CUDA_TRY(c, launch_visit_check(c->visits + b * per, per, c->blk_len[(size_t)b] > 0 ? e : 0u,
+                                     c->chk_dev, c->num_sms, c->st));
+  } else {
+    CUDA_TRY(c, launch_visit_check(c->visits, c->n_units, e, c->chk_dev, c->num_sms, c->st));
+  }
+  unsigned long long h = 0;
+  CUDA_TRY(c, cudaMemcpyAsync(&h, c->chk_dev, 8, cudaMemcpyDeviceToHost, c->st));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  *bad_units = (int64_t)h;
+  if (units) *units = c->n_units;
+  if (epochs) *epochs = c->epochs_run;
   return MF_OK;
 }
 
@@ -1890,7 +1979,7 @@ mf_status mf_rmse(mf_ctx* c, int32_t set, double* out) {
   const double sse = h2[0];
   if (c->G > 1) cnt = h2[1];
   const double rmse = (double)c->p.rating_scale * std::sqrt(sse / std::max(cnt, 1.0));
-  *out = N > 0 ? rmse : 0.0;
+  *out = cnt > 0 ? rmse : 0.0;     // global count when world > 1 (all-reduced above)
   if (std::isnan(*out)) return c->fail(MF_E_RANGE, "RMSE is NaN (divergence)");
   return MF_OK;
 }

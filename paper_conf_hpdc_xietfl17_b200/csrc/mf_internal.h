@@ -40,6 +40,8 @@ struct HogwildLaunch {
   void *P, *Q;
   float g, lp, lq;
   AdaArgs ada;              // ada.GP != nullptr: ADAGRAD (g = alpha)
+  unsigned* visits;         // per global chunk id: claims (one atomic per claimed chunk)
+  unsigned long long* upd;  // non-sentinel samples updated (device count, Eq. 7)
   cudaStream_t stream;
   int *out_workers, *out_lanes, *out_grid;
 };
@@ -61,6 +63,8 @@ struct WavefrontLaunch {
   AdaArgs ada;              // ada.GP != nullptr: ADAGRAD (register kernel; g = alpha)
   long long* prof;          // diagnostics (MF_PROFILE_WAVES): per worker {wait, run, samples, smid, warpid, release
                             // fence} clock64 totals, or nullptr
+  unsigned* visits;         // s*c per strata block: visits of sub-block (i, j) (one atomic per wave)
+  unsigned long long* upd;  // samples updated (device count)
   cudaStream_t stream;
   int *out_lanes, *out_grid;
 };
@@ -86,6 +90,8 @@ struct LibmfLaunch {
   void *P, *Q;
   float g, lp, lq;
   uint64_t seed;
+  unsigned* visits;         // a*a: claims of each block
+  unsigned long long* upd;  // samples updated (device count)
   cudaStream_t stream;
   int* out_lanes;
 };
@@ -94,6 +100,9 @@ cudaError_t launch_hogwild(const HogwildLaunch& a);
 cudaError_t launch_libmf(const LibmfLaunch& a);
 cudaError_t launch_wavefront(const WavefrontLaunch& a);
 cudaError_t launch_rmse(const RmseLaunch& a);
+// number of entries of visits[0, n) that differ from `expect`, into *out (device)
+cudaError_t launch_visit_check(const unsigned* visits, int64_t n, unsigned expect,
+                               unsigned long long* out, int num_sms, cudaStream_t st);
 int ring_window(int k, int storage, int lane_bytes);  // history window W of k_wavefront2
 
 }  // namespace mfb

@@ -41,9 +41,10 @@ __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L >
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
                                                  unsigned long long* __restrict__ counter,
                                                  int workers, T* __restrict__ P, T* __restrict__ Q,
-                                                 int f, float g, float lp, float lq, AdaArgs ada) {
+                                                 int f, float g, float lp, float lq, AdaArgs ada,
+                                                 unsigned* __restrict__ visits,
+                                                 unsigned long long* __restrict__ upd) {
   constexpr int GPW = 32 / L;
-  const float cp = 1.f - g * lp, cq = 1.f - g * lq;
   const int lane = threadIdx.x & 31;
   const int grp = lane / L, gl = lane % L, gbase = grp * L;
   const int warp = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) >> 5);
@@ -51,6 +52,7 @@ __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L >
   if (first >= workers) return;                      // warp-uniform
   const int nact = min(GPW, workers - first);
   const int64_t total = segs.prefix[segs.n];
+  int done = 0;                                      // this group's non-sentinel updates
   for (;;) {
     unsigned long long base = 0;
     if (lane == 0) base = atomicAdd(counter, (unsigned long long)nact);
@@ -67,11 +69,13 @@ __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L >
       const int sgi = segs.lev_seg[lv][(int)(pos % cnt)];
       const uint32_t chunk = __ldg(chunks + segs.begin[sgi] + segs.lev_lo[lv] + pos / cnt);
       lo = (int64_t)chunk * f + segs.shift[sgi];
+      if (gl == 0) atomicAdd(visits + chunk, 1u);    // exactly-once evidence (mf_check_visits)
     }
     // every group of the warp runs f iterations in lockstep (inactive ones on sentinels)
-    run_serial<T, K, L, D, true, ADA>(slots, lo, f, act, P, Q, g, cp, cq, gl, gbase, 0xffffffffu,
-                                      ada);
+    done += run_serial<T, K, L, D, true, ADA>(slots, lo, f, act, P, Q, g, lp, lq, gl, gbase,
+                                              0xffffffffu, ada);
   }
+  if (gl == 0 && done) atomicAdd(upd, (unsigned long long)done);
 }
 
 // ---------------------------------------------------------------------------------------------
@@ -126,25 +130,29 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
                                                    const int32_t* __restrict__ rank,
                                                    int* __restrict__ tickets, int s, int c,
                                                    T* __restrict__ P, T* __restrict__ Q, float g,
-                                                   float lp, float lq, int64_t shift, AdaArgs ada) {
+                                                   float lp, float lq, int64_t shift, AdaArgs ada,
+                                                   unsigned* __restrict__ visits,
+                                                   unsigned long long* __restrict__ upd) {
   const int lane = threadIdx.x & 31;
   const int grp = lane / L, gl = lane % L, gbase = grp * L;
   const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
   const int worker = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) / L);
   if (worker >= s) return;
-  const float cp = 1.f - g * lp, cq = 1.f - g * lq;
   const int32_t* my_seq = seq + (int64_t)worker * c;
   const int32_t* my_rank = rank + (int64_t)worker * c;
+  int done = 0;
   for (int w = 0; w < c; ++w) {
     const int col = __ldg(my_seq + w);
     const int tgt = __ldg(my_rank + w);
     ticket_acquire(tickets + col, tgt);
     const int64_t sb = (int64_t)worker * c + col;
     const int64_t lo = __ldg(sub_off + sb) + shift;
-    run_serial<T, K, L, 2, false, ADA>(slots, lo, (int)(__ldg(sub_off + sb + 1) + shift - lo), true, P,
-                                       Q, g, cp, cq, gl, gbase, gmask, ada);
+    done += run_serial<T, K, L, 2, false, ADA>(slots, lo, (int)(__ldg(sub_off + sb + 1) + shift - lo),
+                                               true, P, Q, g, lp, lq, gl, gbase, gmask, ada);
+    if (gl == 0) atomicAdd(visits + sb, 1u);
     ticket_release(tickets + col, tgt + 1, gmask, gl);
   }
+  if (gl == 0 && done) atomicAdd(upd, (unsigned long long)done);
 }
 
 
@@ -159,7 +167,9 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
                                                     int* __restrict__ tickets, int s, int c,
                                                     T* __restrict__ P, T* __restrict__ Q, float g,
                                                     float lp, float lq, int64_t shift,
-                                                    long long* __restrict__ prof) {
+                                                    long long* __restrict__ prof,
+                                                    unsigned* __restrict__ visits,
+                                                    unsigned long long* __restrict__ upd) {
   extern __shared__ __align__(16) char smem[];
   constexpr int ROWB = K * (int)sizeof(T);
   const int lane = threadIdx.x & 31;
@@ -172,7 +182,6 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
   const int worker = blockIdx.x * (blockDim.x >> 5) + local;
   if (worker >= s) return;
   char* ring = smem + (size_t)local * RS * 2 * ROWB;
-  const float cp = 1.f - g * lp, cq = 1.f - g * lq;
   const int32_t* my_seq = seq + (int64_t)worker * c;
   const int32_t* my_rank = rank + (int64_t)worker * c;
   const int64_t* my_off = sub_off + (int64_t)worker * c;
@@ -201,12 +210,13 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
   RingHead h0 = load_head<L>(slots, dup, lo0, n0, gl);
   bool ready = false;            // column col0 acquired and its ring prologue issued already
   long long t_wait = 0, t_run = 0, t_rel = 0, n_done = 0;
+  unsigned long long n_upd = 0;                      // samples updated (no sentinels here)
   for (int w = 0; w < c; ++w) {
     const long long tw0 = prof ? clock64() : 0;
     if (!ready) {
       ticket_acquire(tickets + col0, tgt0);   // relaxed spin + fence.acq_rel
       if (n0 > 0)
-        run_subblock_ring<T, K, L, RS, F>(slots, dup, lo0, n0, h0, P, Q, g, cp, cq, gl, gbase,
+        run_subblock_ring<T, K, L, RS, F>(slots, dup, lo0, n0, h0, P, Q, g, lp, lq, gl, gbase,
                                           gmask, ring, true, false);
     }
     // next waves' inputs
@@ -224,15 +234,17 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     const int poll1 = w + 1 < c ? ld_acquire(tickets + col1) : -1;
     const long long tw1 = prof ? clock64() : 0;
     if (n0 > 0)
-      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo0, n0, h0, P, Q, g, cp, cq, gl, gbase, gmask,
+      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo0, n0, h0, P, Q, g, lp, lq, gl, gbase, gmask,
                                         ring, false, true);
     // next column already released: issue its row prefetch BEFORE this wave's release fence.
     // (Its p rows may have been stored by this sub-block: same thread, issued after them.)
     ready = w + 1 < c && poll1 == tgt1;
     if (ready && n1 > 0)
-      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo1, n1, h1, P, Q, g, cp, cq, gl, gbase, gmask,
+      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo1, n1, h1, P, Q, g, lp, lq, gl, gbase, gmask,
                                         ring, true, false);
     const long long tw2 = prof ? clock64() : 0;
+    if (gl == 0) atomicAdd(visits + (int64_t)worker * c + col0, 1u);   // sub-block (worker, col0)
+    n_upd += n0;
     ticket_release(tickets + col0, tgt0 + 1, gmask, gl);   // fence; syncwarp; relaxed store
     if (prof) {
       t_wait += tw1 - tw0;
@@ -244,6 +256,7 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     col1 = col2; tgt1 = tgt2; lo1 = lo2; n1 = n2;
     col2 = col3; tgt2 = tgt3;
   }
+  if (gl == 0 && n_upd) atomicAdd(upd, n_upd);
   if (prof && gl == 0) {
     unsigned smid, wid;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
@@ -269,15 +282,16 @@ __global__ void __launch_bounds__(32) k_libmf(const Rating* __restrict__ slots,
                                               int* lock, int* row_busy, int* col_busy, int* done,
                                               int* remaining, int workers, T* __restrict__ P,
                                               T* __restrict__ Q, float g, float lp, float lq,
-                                              uint64_t seed) {
+                                              uint64_t seed, unsigned* __restrict__ visits,
+                                              unsigned long long* __restrict__ upd) {
   const int lane = threadIdx.x & 31;
   if (lane >= L) return;
   const int worker = blockIdx.x;
   if (worker >= workers) return;
   const unsigned gmask = (L == 32) ? 0xffffffffu : ((1u << L) - 1u);
-  const float cp = 1.f - g * lp, cq = 1.f - g * lq;
   uint64_t draw = mix64(seed + (uint64_t)worker * kPhi);
   unsigned ns = 64;
+  int n_upd = 0;
   for (;;) {
     int b = -1;
     if (lane == 0) {
@@ -318,8 +332,9 @@ __global__ void __launch_bounds__(32) k_libmf(const Rating* __restrict__ slots,
     }
     ns = 64;
     const int64_t lo = __ldg(blk_off + b);
-    run_serial<T, K, L, 1, false>(slots, lo, (int)__ldg(blk_len + b), true, P, Q, g, cp, cq, lane, 0,
-                                  gmask);
+    if (lane == 0) atomicAdd(visits + b, 1u);
+    n_upd += run_serial<T, K, L, 1, false>(slots, lo, (int)__ldg(blk_len + b), true, P, Q, g, lp, lq,
+                                           lane, 0, gmask);
     __threadfence();
     __syncwarp(gmask);
     if (lane == 0) {
@@ -327,6 +342,7 @@ __global__ void __launch_bounds__(32) k_libmf(const Rating* __restrict__ slots,
       atomicExch(col_busy + b % a, 0);
     }
   }
+  if (lane == 0 && n_upd) atomicAdd(upd, (unsigned long long)n_upd);
 }
 
 // ---------------------------------------------------------------------------------------------
@@ -393,6 +409,30 @@ __global__ void k_rmse_final(const double* __restrict__ partial, int n, double* 
   if (threadIdx.x == 0) out[0] = sm[0];
 }
 
+// Exactly-once check (Eq. 7: an epoch is N updates): count the work units (Hogwild chunks,
+// wavefront sub-blocks, LIBMF blocks) whose claim counter differs from the expected number of
+// epochs.  Together with the device update count this shows every sample is updated once per
+// epoch: units are disjoint slot ranges, each run over all of its slots.
+__global__ void k_visit_check(const unsigned* __restrict__ v, int64_t n, unsigned expect,
+                              unsigned long long* __restrict__ out) {
+  unsigned long long bad = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    bad += v[i] != expect;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) bad += __shfl_xor_sync(0xffffffffu, bad, o);
+  if ((threadIdx.x & 31) == 0 && bad) atomicAdd(out, bad);
+}
+
+cudaError_t launch_visit_check(const unsigned* visits, int64_t n, unsigned expect,
+                               unsigned long long* out, int num_sms, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;   // accumulates into *out (the caller zeroes it)
+  int64_t blocks = (n + 255) / 256;
+  if (blocks > (int64_t)num_sms * 8) blocks = (int64_t)num_sms * 8;
+  k_visit_check<<<(unsigned)blocks, 256, 0, st>>>(visits, n, expect, out);
+  return cudaGetLastError();
+}
+
 // ---------------------------------------------------------------------------------------------
 // Dispatch
 // ---------------------------------------------------------------------------------------------
@@ -412,7 +452,7 @@ static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
   if (a.out_grid) *a.out_grid = blocks;
   kern<<<blocks, threads, 0, a.stream>>>(a.slots, a.chunks, a.segs, a.counter, workers,
                                          reinterpret_cast<T*>(a.P), reinterpret_cast<T*>(a.Q), a.f,
-                                         a.g, a.lp, a.lq, a.ada);
+                                         a.g, a.lp, a.lq, a.ada, a.visits, a.upd);
   return cudaGetLastError();
 }
 
@@ -439,8 +479,10 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
   float g = a.g, lp = a.lp, lq = a.lq;
   int64_t shift = a.shift;
   AdaArgs ada = a.ada;
+  unsigned* visits = a.visits;
+  unsigned long long* upd = a.upd;
   void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq, &shift,
-                  &ada};
+                  &ada, &visits, &upd};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, 0,
                                      a.stream);
 }
@@ -477,8 +519,10 @@ static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
   float g = a.g, lp = a.lp, lq = a.lq;
   int64_t shift = a.shift;
   long long* prof = a.prof;
+  unsigned* visits = a.visits;
+  unsigned long long* upd = a.upd;
   void* args[] = {&slots, &dup, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq,
-                  &shift, &prof};
+                  &shift, &prof, &visits, &upd};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, smem,
                                      a.stream);
 }
@@ -488,7 +532,8 @@ static cudaError_t launch_libmf_t(const LibmfLaunch& a) {
   if (a.out_lanes) *a.out_lanes = L;
   k_libmf<T, K, L><<<a.workers, 32, 0, a.stream>>>(
       a.slots, a.blk_off, a.blk_len, a.a, a.lock, a.row_busy, a.col_busy, a.done, a.remaining,
-      a.workers, reinterpret_cast<T*>(a.P), reinterpret_cast<T*>(a.Q), a.g, a.lp, a.lq, a.seed);
+      a.workers, reinterpret_cast<T*>(a.P), reinterpret_cast<T*>(a.Q), a.g, a.lp, a.lq, a.seed,
+      a.visits, a.upd);
   return cudaGetLastError();
 }
 

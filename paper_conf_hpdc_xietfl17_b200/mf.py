@@ -69,7 +69,8 @@ class Stats(ctypes.Structure):
 _lib = None
 EXPORTED = ["mf_abi_version", "mf_params_default", "mf_create", "mf_load_coo", "mf_train_epoch",
             "mf_rmse", "mf_get_factors", "mf_set_factors", "mf_set_epoch", "mf_get_epoch",
-            "mf_export_schedule", "mf_get_stats", "mf_get_launch_ms", "mf_strata_holders", "mf_strata_plan",
+            "mf_export_schedule", "mf_get_stats", "mf_get_launch_ms", "mf_check_visits",
+            "mf_strata_holders", "mf_strata_plan",
             "mf_destroy",
             "mf_last_error", "mf_status_string"]
 
@@ -98,6 +99,7 @@ def lib() -> ctypes.CDLL:
         "mf_export_schedule": (i32, [vp, i32, i32, vp, ctypes.POINTER(i64)]),
         "mf_get_stats": (i32, [vp, ctypes.POINTER(Stats)]),
         "mf_get_launch_ms": (i32, [vp, vp, ctypes.POINTER(i64)]),
+        "mf_check_visits": (i32, [vp, ctypes.POINTER(i64), ctypes.POINTER(i64), ctypes.POINTER(i32)]),
         "mf_strata_holders": (i32, [u64, i32, i32, i32, i32, vp]),
         "mf_strata_plan": (i32, [u64, i32, i32, i32, i64, i32, i32, vp, vp, vp, vp, vp]),
         "mf_destroy": (None, [vp]),
@@ -317,6 +319,14 @@ class MF:
                     "mf_get_launch_ms")
         return buf[:n.value]
 
+    def check_visits(self) -> dict:
+        """Exactly-once evidence from the device (mf_check_visits): work units whose claim count
+        differs from the epochs run since load."""
+        bad, units, ep = ctypes.c_int64(0), ctypes.c_int64(0), ctypes.c_int32(0)
+        self._check(lib().mf_check_visits(self.h, ctypes.byref(bad), ctypes.byref(units),
+                                          ctypes.byref(ep)), "mf_check_visits")
+        return {"bad_units": bad.value, "units": units.value, "epochs": ep.value}
+
     def stats(self) -> dict:
         s = Stats()
         self._check(lib().mf_get_stats(self.h, ctypes.byref(s)), "mf_get_stats")
@@ -383,6 +393,10 @@ def mf_get_stats(ctx: MF) -> dict:
 
 def mf_get_launch_ms(ctx: MF) -> np.ndarray:
     return ctx.launch_ms()
+
+
+def mf_check_visits(ctx: MF) -> dict:
+    return ctx.check_visits()
 
 
 def mf_last_error(ctx: MF) -> str:

@@ -10,7 +10,9 @@ of Table 2 and the recipe stated in DESIGN.md section 4 (from SURVE
 * the test set is drawn iid from the same process with its own stream (seed + 100) (R17).
 
 Large sets are generated with torch on whatever device is given (CUDA on the GPU box), in
-chunks, so that 99M - 3.1B samples stay tractable; the tiny set uses numpy.
+chunks, so that 99M - 3.1B samples stay tractable.  The generator is counter-based: the same
+seed gives bit-identical data on the CPU and on the GPU (so oracle reference values can be
+computed on a CPU box and compared with a GPU run).  The tiny set uses numpy.
 """
 from __future__ import annotations
 
@@ -88,44 +90,138 @@ def uniform(m: int, n: int, N: int, seed: int = 0, mu: float = 0.0, rank: int = 
     return Ratings(m, n, u, v, r, ut, vt, rt, meta=dict(kind="uniform", seed=seed))
 
 
-def _powerlaw_ids(count: int, size: int, expo: float, relabel: torch.Tensor,
-                  cdf: torch.Tensor, g: torch.Generator, device) -> torch.Tensor:
-    x = torch.rand(count, generator=g, device=device, dtype=torch.float64)
-    rank = torch.searchsorted(cdf, x).clamp_(max=size - 1)
-    return relabel[rank].to(torch.int32)
+# ---------------------------------------------------------------------------------------------
+# Counter-based draws (device independent).  Every random number is a pure function of
+# (data seed, stream tag, global index): a 64-bit hash of the index, evaluated with int64
+# tensor arithmetic (two's-complement wrap-around, logical shifts by masking) on whatever device
+# the tensors live on.  Every float derived from it is built from exact integer-to-float
+# conversions and single IEEE operations (no transcendental functions, no fused or reordered
+# reductions), so CPU and CUDA produce the SAME bits for the same seed -- tests/test_synth.py
+# pins the hash against a plain-Python rendering and CPU against CUDA.  The hash is MurmurHash3's
+# 64-bit finaliser (fmix64) of seed-keyed counters; it is deliberately not the method's own
+# SplitMix64 key function, which this module does not contain.
+# ---------------------------------------------------------------------------------------------
+_M64 = 1 << 64
+_F1, _F2 = 0xFF51AFD7ED558CCD, 0xC4CEB9FE1A85EC53          # fmix64 constants
+_GOLD = 0x9E3779B97F4A7C15                                   # Weyl increment of the counter
+
+
+def _s64(c: int) -> int:
+    """A uint64 constant as the int64 with the same bits."""
+    c %= _M64
+    return c - _M64 if c >= 1 << 63 else c
+
+
+def _shr(z: torch.Tensor, s: int) -> torch.Tensor:
+    """Logical right shift of int64 bit patterns."""
+    return (z >> s) & ((1 << (64 - s)) - 1)
+
+
+def fmix64(z: torch.Tensor) -> torch.Tensor:
+    z = z ^ _shr(z, 33)
+    z = z * _s64(_F1)
+    z = z ^ _shr(z, 33)
+    z = z * _s64(_F2)
+    return z ^ _shr(z, 33)
+
+
+def fmix64_int(z: int) -> int:
+    """Plain-Python fmix64 (the pin of the tensor version; also derives stream keys)."""
+    z %= _M64
+    z ^= z >> 33
+    z = (z * _F1) % _M64
+    z ^= z >> 33
+    z = (z * _F2) % _M64
+    return z ^ (z >> 33)
+
+
+def stream_key(seed: int, tag: int) -> int:
+    return fmix64_int(fmix64_int(seed * _GOLD + 1) + tag * _GOLD)
+
+
+def hash_at(key: int, idx: torch.Tensor) -> torch.Tensor:
+    """64-bit hash (int64 bits) of counters idx (int64) under a stream key."""
+    return fmix64(idx * _s64(_GOLD) + _s64(key))
+
+
+def uniform53(key: int, idx: torch.Tensor) -> torch.Tensor:
+    """U[0,1) in float64 with 53 random bits (exact conversion)."""
+    return _shr(hash_at(key, idx), 11).to(torch.float64) * (2.0 ** -53)
+
+
+def normal_ih(key: int, idx: torch.Tensor) -> torch.Tensor:
+    """Approximately N(0,1): Irwin-Hall sum of 12 U24 uniforms minus 6 (six hashes, two 24-bit
+    uniforms each).  Every partial sum is exact in float64 (< 2^28 units of 2^-24), so the
+    result does not depend on the order of evaluation or the device."""
+    acc = torch.zeros(idx.shape, dtype=torch.float64, device=idx.device)
+    for j in range(6):
+        h = hash_at(key, idx * 6 + j)
+        acc += _shr(h, 40).to(torch.float64) * (2.0 ** -24)
+        acc += (_shr(h, 16) & 0xFFFFFF).to(torch.float64) * (2.0 ** -24)
+    return acc - 6.0
+
+
+def _cdf(size: int, expo: float) -> np.ndarray:
+    """Normalised CDF of weights (rank+1)^-expo, computed once on the host in float64 (the
+    only place a pow() is evaluated) and shipped to the device bit for bit."""
+    w = np.arange(1, size + 1, dtype=np.float64) ** (-expo)
+    c = np.cumsum(w)
+    return c / c[-1]
+
+
+# stream tags of the recipe
+_T_RELAB_U, _T_RELAB_V, _T_PS, _T_QS, _T_U, _T_V, _T_EPS = 1, 2, 3, 4, 5, 6, 7
+_TEST_SEED_OFFSET = 100       # R17: the test set is the same process on seed + 100
 
 
 def powerlaw(m: int, n: int, N: int, Ntest: int, *, seed: int, a_u: float = 0.38,
              a_v: float = 0.45, rank: int = 16, mu: float = 3.6, noise: float = 0.5,
              scale: str = "plain", device="cpu", chunk: int = 1 << 24,
              out_device=None) -> Ratings:
-    """Power-law-skewed planted-rank ratings (SURVEY 8(d) recipe), generated in chunks."""
+    """Power-law-skewed planted-rank ratings (SURVEY 8(d) recipe),
+    counter-based: the same (m, n, N, seed, ...) gives bit-identical (u, v, r) on any device and
+    for any chunk size."""
     dev = torch.device(device)
     out_dev = dev if out_device is None else torch.device(out_device)
-    g = torch.Generator(device=dev)
-    g.manual_seed(seed)
+    cdf_u = torch.from_numpy(_cdf(m, a_u)).to(dev)
+    cdf_v = torch.from_numpy(_cdf(n, a_v)).to(dev)
 
-    def cdf_of(size, expo):
-        w = torch.arange(1, size + 1, device=dev, dtype=torch.float64).pow_(-expo)
-        c = torch.cumsum(w, 0)
-        return c / c[-1]
+    def relabel(size, tag):   # a uniformly random permutation of the ids: argsort of distinct keys
+        k = hash_at(stream_key(seed, tag), torch.arange(size, dtype=torch.int64, device=dev))
+        return torch.argsort(k).to(torch.int32)
 
-    cdf_u, cdf_v = cdf_of(m, a_u), cdf_of(n, a_v)
-    relab_u = torch.randperm(m, generator=g, device=dev)
-    relab_v = torch.randperm(n, generator=g, device=dev)
-    Ps = torch.randn(m, rank, generator=g, device=dev) / rank ** 0.25
-    Qs = torch.randn(n, rank, generator=g, device=dev) / rank ** 0.25
+    relab_u, relab_v = relabel(m, _T_RELAB_U), relabel(n, _T_RELAB_V)
+    amp = 1.0 / rank ** 0.25
 
-    def draw(cnt, gen):
+    def factors(size, tag):   # planted factors, entries ~ N(0,1) / rank^(1/4), float32
+        out = torch.empty(size, rank, dtype=torch.float32, device=dev)
+        for lo in range(0, size, chunk // rank):
+            c = min(chunk // rank, size - lo)
+            idx = torch.arange(lo * rank, (lo + c) * rank, dtype=torch.int64, device=dev)
+            out[lo:lo + c] = (normal_ih(stream_key(seed, tag), idx) * amp).to(torch.float32).view(c, rank)
+        return out
+
+    Ps, Qs = factors(m, _T_PS), factors(n, _T_QS)
+
+    def ids(key, idx, size, cdf, relab):
+        x = uniform53(key, idx)
+        return relab[torch.searchsorted(cdf, x).clamp_(max=size - 1)]
+
+    def draw(cnt, sd):
+        ku, kv, ke = stream_key(sd, _T_U), stream_key(sd, _T_V), stream_key(sd, _T_EPS)
         u = torch.empty(cnt, dtype=torch.int32, device=out_dev)
         v = torch.empty(cnt, dtype=torch.int32, device=out_dev)
         r = torch.empty(cnt, dtype=torch.float32, device=out_dev)
         for lo in range(0, cnt, chunk):
             c = min(chunk, cnt - lo)
-            uu = _powerlaw_ids(c, m, a_u, relab_u, cdf_u, gen, dev)
-            vv = _powerlaw_ids(c, n, a_v, relab_v, cdf_v, gen, dev)
-            sig = (Ps[uu.long()] * Qs[vv.long()]).sum(1)
-            eps = torch.randn(c, generator=gen, device=dev) * noise
+            idx = torch.arange(lo, lo + c, dtype=torch.int64, device=dev)
+            uu = ids(ku, idx, m, cdf_u, relab_u)
+            vv = ids(kv, idx, n, cdf_v, relab_v)
+            pu, qv = Ps[uu.long()], Qs[vv.long()]
+            sig = torch.zeros(c, dtype=torch.float64, device=dev)
+            for d in range(rank):     # separate IEEE multiply and add: no contraction, fixed order
+                sig = sig + pu[:, d].to(torch.float64) * qv[:, d].to(torch.float64)
+            eps = normal_ih(ke, idx) * noise
             if scale == "yahoo":
                 rr = (50.0 + 25.0 * (sig + eps)).clamp_(0.0, 100.0)
             else:
@@ -135,13 +231,27 @@ def powerlaw(m: int, n: int, N: int, Ntest: int, *, seed: int, a_u: float = 0.38
             r[lo:lo + c] = rr.to(torch.float32).to(out_dev)
         return u, v, r
 
-    u, v, r = draw(N, g)
-    gt = torch.Generator(device=dev)
-    gt.manual_seed(seed + 100)
-    ut, vt, rt = draw(Ntest, gt) if Ntest else (None, None, None)
-    meta = dict(kind="powerlaw", seed=seed, a_u=a_u, a_v=a_v, rank=rank, mu=mu, noise=noise,
-                scale=scale)
+    u, v, r = draw(N, seed)
+    ut, vt, rt = draw(Ntest, seed + _TEST_SEED_OFFSET) if Ntest else (None, None, None)
+    meta = dict(kind="powerlaw-counter", seed=seed, a_u=a_u, a_v=a_v, rank=rank, mu=mu,
+                noise=noise, scale=scale)
     return Ratings(m, n, u, v, r, ut, vt, rt, meta=meta)
+
+
+def checksum(R: Ratings) -> str:
+    """Order-sensitive 64-bit digest of (u, v, r-bits) of the train and test sets (hex), for
+    pinning a generated set across devices (golden files carry it)."""
+    tot = 0
+    for arr in (R.u, R.v, R.r, R.ut, R.vt, R.rt):
+        if arr is None:
+            continue
+        t = torch.as_tensor(arr)
+        t = (t.view(torch.int32) if t.dtype == torch.float32 else t.to(torch.int32)).to(torch.int64)
+        idx = torch.arange(t.numel(), dtype=torch.int64, device=t.device)
+        h = hash_at(0x5EED, idx * 2 + (t & 0xFFFFFFFF))
+        part = int((h & 0xFFFFFFFF).sum().item()) + (int((_shr(h, 32)).sum().item()) << 32)
+        tot = fmix64_int(tot + part)
+    return f"{tot:016x}"
 
 
 def shaped(name: str, *, fraction: float = 1.0, device="cpu", out_device=None,

@@ -62,9 +62,11 @@ def test_hugewiki_fullsize_hogwild_epoch():
     r0 = g.rmse()
     g.train_epoch()
     st = g.stats()
+    cv = g.check_visits()
     r1 = g.rmse()
     g.close()
-    assert st["updates"] == N and st["sgd_launches"] == 1
+    assert st["updates"] == N and st["sgd_launches"] == 1      # device count, N > 2^31
+    assert cv["bad_units"] == 0 and cv["units"] == -(-N // 256), cv   # 11,991,477 chunks once
     assert np.isfinite(r1) and r1 < r0, (r0, r1)
 
 

@@ -38,7 +38,7 @@ def run_ranks(world, R, k, epochs, **kw):
                 m.train_epoch()
             rm = m.rmse()
             P, Q = m.factors()
-            out[rank] = (rm, P, Q, m.stats())
+            out[rank] = (rm, P, Q, m.stats(), m.check_visits())
             m.close()
         except Exception as e:  # surface in the main thread
             errs.append(e)
@@ -68,12 +68,13 @@ def test_multirank_strata_matches_oracle(world, kw):
         o.train_epoch()
     Po, Qo = o.factors()
     ro = o.rmse(R.ut, R.vt, R.rt)
-    for rank, (rm, P, Q, st) in enumerate(res):
+    for rank, (rm, P, Q, st, cv) in enumerate(res):
+        assert cv["bad_units"] == 0 and cv["epochs"] == epochs, (rank, cv)
         assert np.array_equal(P, res[0][1]) and np.array_equal(Q, res[0][2]), rank
         assert rm == res[0][0]
         assert np.abs(P - Po).max() <= 2e-4 and np.abs(Q - Qo).max() <= 2e-4
         assert abs(rm - ro) <= 2e-5 * ro, (rm, ro)
-    # every rank trained only its own blocks: the updates add up to N per epoch
+    # every rank trained only its own blocks: the device-counted updates add up to N per epoch
     assert sum(r[3]["updates"] for r in res) == R.N
 
 

@@ -130,13 +130,17 @@ def test_deterministic_parity_other_k_ragged(k, wfk, lb):
 @pytest.mark.parametrize("storage,k,lb", [("fp16", 16, 0), ("bf16", 16, 0), ("fp16", 128, 0),
                                          ("bf16", 128, 0), ("fp16", 128, 16)])
 def test_deterministic_parity_low_precision_storage(tiny, storage, k, lb):
-    """Storage rounding is RNE on both sides (R16), but the fp32 value being rounded
-    differs between the two sides by the dot-product order (tree vs sequential, ~k*eps32), so an
-    update can round to the neighbouring storage value: one ulp of that value's binade, which
-    later updates carry along as an ABSOLUTE offset (damped by gamma).  Bar: every entry within
-    2 ulps of the largest binade in use (absolute), >75% of entries identical, test RMSE within
-    1e-4 relative.  k = 128 runs the ring kernel on the ragged set: lb = 0
-    is its default 32-lane geometry (8-B lane slices, split row copy), lb = 16 the 16-lane one."""
+    """Storage rounding is RNE on both sides (R16) and the kernel evaluates lines 9-10
+    in the paper's operation order (mf_sgd.cuh sgd_update), so the fp32 value being rounded
+    differs from the oracle's only through the dot product's summation order (lane partials and
+    a group sum vs a sequential sum, ~k*eps32 relative).  An update whose value lies within that
+    of a rounding boundary stores the neighbouring storage value: one ulp of its binade, which
+    later updates carry along as an ABSOLUTE offset (damped by gamma).  A CPU emulation of both
+    operation orders on the tiny set leaves 99.98-99.99% of the entries
+    identical (the earlier 2-op update form: ~90%).  Bar: >99% identical, every entry within
+    2 ulps of the largest binade in use (absolute), test RMSE within 1e-4 relative.  k = 128 runs
+    the ring kernel on the ragged set: lb = 0 is its default 32-lane geometry (8-B lane slices),
+    lb = 16 the 16-lane one."""
     R = tiny if k == 16 else ragged()
     g, o = pair(R, k=k, storage=storage, schedule="wavefront", workers=8 if k == 16 else 6,
                 wf_cols=16 if k == 16 else 9, lane_bytes=lb, **TABLE3_NETFLIX)
@@ -147,7 +151,7 @@ def test_deterministic_parity_low_precision_storage(tiny, storage, k, lb):
     for Xg, Xo in zip(g.factors(), o.factors()):
         ulp_abs = 2.0 ** (np.floor(np.log2(np.abs(Xo).max())) - mant)
         diag = (storage, float(np.mean(Xg == Xo)), float(np.abs(Xg - Xo).max()), ulp_abs, rg, ro)
-        assert np.mean(Xg == Xo) > 0.75, diag
+        assert np.mean(Xg == Xo) > 0.99, diag
         assert np.abs(Xg - Xo).max() <= 2 * ulp_abs, diag
     assert abs(rg - ro) <= 1e-4 * ro, (rg, ro)
 
@@ -197,6 +201,72 @@ def test_hogwild_powerlaw_20_epochs_matches_oracle():
     assert abs(rg - ro) <= 0.005 * ro, (rg, ro)
 
 
+@pytest.mark.parametrize("storage,k,lb", [("fp32", 128, 0), ("fp16", 128, 0), ("bf16", 128, 0),
+                                         ("fp32", 32, 0), ("fp32", 64, 0), ("fp32", 256, 0),
+                                         ("fp16", 32, 0), ("fp16", 64, 0), ("fp16", 256, 0),
+                                         ("fp32", 128, 32), ("fp16", 128, 8)])
+def test_hogwild_one_worker_elementwise_parity_all_k(storage, k, lb):
+    """The bench's kernel instantiations at 1 worker (= the oracle's serial batch-Hogwild order,
+    R7): k_hogwild<__half,128,16> (the headline configuration), <float,128,32>, bf16, and
+    k = 32/64/256, on the ragged set (N = 12,345: chunks of 256 with a ragged last chunk, odd m,
+    n, duplicate pairs), 2 epochs.  fp32: |dP|, |dQ| <= 1e-4 and RMSE relative <= 1e-5;
+    fp16/bf16: the low-precision bar of test_deterministic_parity_low_precision_storage."""
+    R = ragged()
+    g, o = pair(R, k=k, storage=storage, schedule="hogwild", workers=1, lane_bytes=lb,
+                **TABLE3_NETFLIX)
+    for _ in range(2):
+        g.train_epoch()
+        o.train_epoch()
+    assert g.stats()["updates"] == R.N
+    rg, ro = g.rmse(), o.rmse(R.ut, R.vt, R.rt)
+    if storage == "fp32":
+        for Xg, Xo in zip(g.factors(), o.factors()):
+            assert np.abs(Xg - Xo).max() <= 1e-4
+        assert abs(rg - ro) <= 1e-5 * ro, (rg, ro)
+        return
+    mant = 10 if storage == "fp16" else 7
+    for Xg, Xo in zip(g.factors(), o.factors()):
+        ulp_abs = 2.0 ** (np.floor(np.log2(np.abs(Xo).max())) - mant)
+        diag = (storage, k, float(np.mean(Xg == Xo)), float(np.abs(Xg - Xo).max()), ulp_abs)
+        assert np.mean(Xg == Xo) > 0.99, diag
+        assert np.abs(Xg - Xo).max() <= 2 * ulp_abs, diag
+    assert abs(rg - ro) <= 1e-4 * ro, (rg, ro)
+
+
+def test_appendix_a_hand_pins_through_the_abi(golden_dir):
+    """The hand-derived App. A values of tests/golden/appendix_a_blocks.json (relabel ranks,
+    strata blocks, wavefront sub-blocks with ragged segments, cyclic sequences and tickets)
+    through mf_export_schedule, and the N = 10 storage order against perm_S_SHUF_10."""
+    import json
+    import os
+    with open(os.path.join(golden_dir, "appendix_a_blocks.json")) as f:
+        g = json.load(f)
+    with open(os.path.join(golden_dir, "appendix_a.json")) as f:
+        g0 = json.load(f)
+    cs = g["case"]
+    u = np.repeat(np.arange(cs["m"], dtype=np.int32), cs["n"])
+    v = np.tile(np.arange(cs["n"], dtype=np.int32), cs["m"])
+    r = np.ones(cs["N"], np.float32)
+    w = mf.MF(cs["m"], cs["n"], 16, seed=42, grid_a=2, schedule="wavefront", workers=3, wf_cols=4,
+              cyclic=True)
+    w.load(u, v, r)
+    assert w.export("rho_r").tolist() == g["rho_R"] and w.export("rho_c").tolist() == g["rho_C"]
+    blk = np.empty(cs["N"], np.int64)
+    blk[w.export("perm")] = w.export("blockid")
+    assert blk.reshape(cs["m"], cs["n"]).tolist() == g["wavefront_blockid_by_u_v"]
+    assert w.export("wfseq", 0).reshape(12, 4).tolist() == g["cyclic_wfseq_t0"]
+    assert w.export("tickets", 0).reshape(12, 4).tolist() == g["cyclic_tickets_t0"]
+    h = mf.MF(cs["m"], cs["n"], 16, seed=42, grid_a=2)
+    h.load(u, v, r)
+    hb = np.empty(cs["N"], np.int64)
+    hb[h.export("perm")] = h.export("blockid")
+    assert hb.reshape(cs["m"], cs["n"]).tolist() == g["hogwild_blockid_by_u_v"]
+    t = mf.MF(10, 10, 16, seed=42)
+    t.load(np.arange(10, dtype=np.int32), np.arange(10, dtype=np.int32)[::-1].copy(),
+           np.ones(10, np.float32))
+    assert t.export("perm").tolist() == g0["perm_S_SHUF_10"]
+
+
 def test_hogwild_one_worker_reproduces_oracle_curve(tiny):
     """1 worker = the serial batch-Hogwild order of the oracle: the RMSE curve matches epoch by
     epoch -- 1e-5 relative after epoch 1 (north_star), and within 1e-4 over 10 epochs as the
@@ -209,13 +279,38 @@ def test_hogwild_one_worker_reproduces_oracle_curve(tiny):
         assert abs(rg - ro) <= (1e-5 if t == 0 else 1e-4) * ro, (t, rg, ro)
 
 
-def test_hogwild_epoch_updates_every_sample_once(tiny):
+@pytest.mark.parametrize("kw", [dict(schedule="hogwild"), dict(schedule="hogwild", grid_a=8, batch_f=64),
+                                dict(schedule="wavefront", workers=8, wf_cols=16),
+                                dict(schedule="wavefront", workers=8, wf_cols=16, cyclic=True, grid_a=4),
+                                dict(schedule="wavefront", workers=8, wf_cols=16, wf_kernel=2),
+                                dict(schedule="libmf", grid_a=16, workers=4)])
+def test_every_sample_updated_exactly_once_on_the_device(tiny, kw):
+    """Eq. 7: an epoch is N updates.  The kernels count their non-sentinel updates and
+    record one claim per work unit (chunk / sub-block / block) on the device; after E epochs
+    every unit was claimed exactly E times (mf_check_visits) and each epoch updated N samples."""
+    g = mf.MF(tiny.m, tiny.n, 16, **kw)
+    g.load(tiny.u, tiny.v, tiny.r)
+    for e in range(3):
+        g.train_epoch()
+        assert g.stats()["updates"] == tiny.N, (e, kw)
+    cv = g.check_visits()
+    assert cv["bad_units"] == 0 and cv["epochs"] == 3 and cv["units"] > 0, cv
+    st = g.stats()
+    if kw["schedule"] == "hogwild" and "grid_a" not in kw:
+        assert st["sgd_launches"] == 1 and cv["units"] == -(-tiny.N // 256)
+    assert st["bytes_per_update"] == 12 + 4 * 16 * 4
+
+
+def test_visit_check_detects_a_missing_epoch(tiny):
+    """The check is not vacuous: resetting the epoch counter does not reset the claim counts,
+    so a context that ran 2 epochs reports every unit as mismatching if told to expect 0."""
     g = mf.MF(tiny.m, tiny.n, 16)
     g.load(tiny.u, tiny.v, tiny.r)
+    assert g.check_visits()["bad_units"] == 0          # nothing run, nothing claimed
     g.train_epoch()
-    st = g.stats()
-    assert st["updates"] == tiny.N and st["sgd_launches"] == 1
-    assert st["bytes_per_update"] == 12 + 4 * 16 * 4
+    g.train_epoch()
+    cv = g.check_visits()
+    assert cv["bad_units"] == 0 and cv["epochs"] == 2
 
 
 # ----------------------------------------------------------------------------- RMSE / factors
@@ -310,6 +405,46 @@ def test_checkpoint_resume_equals_uninterrupted(tiny):
 
 # ----------------------------------------------------------------------------- out-of-core
 
+@pytest.mark.parametrize("staged", [False, True])
+def test_destroy_right_after_an_epoch_with_the_default_allocator(staged):
+    """an epoch in staged mode ends by queueing the next stratum's H2D copy on the
+    copy stream; mf_destroy must drain it before the stream-ordered frees (cudaMallocAsync
+    allocator, allocator='none')."""
+    R = ragged()
+    for _ in range(3):
+        g = mf.MF(R.m, R.n, 32, staged=staged, grid_a=4, batch_f=64, allocator="none")
+        g.load(R.u, R.v, R.r)
+        g.train_epoch()
+        g.close()
+    torch.cuda.synchronize()
+
+
+def test_failed_load_releases_its_buffers_and_the_ctx_stays_usable():
+    """an MF_E_RANGE load leaves no partial allocation behind; a retried load then
+    succeeds and trains."""
+    R = ragged()
+    g = mf.MF(R.m, R.n, 32, allocator="none")
+    nb = 4 << 20                                       # 48 MB of input copies per attempt
+    rng = np.random.default_rng(1)
+    bu = rng.integers(0, R.m, nb).astype(np.int32)
+    bu[nb // 2] = R.m                                  # one index out of range
+    bv = rng.integers(0, R.n, nb).astype(np.int32)
+    br = np.ones(nb, np.float32)
+    with pytest.raises(mf.MFError):
+        g.load(bu, bv, br)
+    torch.cuda.synchronize()
+    free0 = torch.cuda.mem_get_info()[0]
+    for _ in range(3):
+        with pytest.raises(mf.MFError) as e:
+            g.load(bu, bv, br)
+        assert e.value.status == -6
+    torch.cuda.synchronize()
+    assert free0 - torch.cuda.mem_get_info()[0] < (24 << 20)   # a leak would be >= 144 MB
+    g.load(R.u, R.v, R.r)
+    g.train_epoch()
+    assert g.stats()["updates"] == R.N
+
+
 @pytest.mark.parametrize("kw", [dict(schedule="wavefront", workers=4, wf_cols=5, grid_a=8),
                                 dict(schedule="wavefront", workers=4, wf_cols=5, grid_a=1),
                                 dict(schedule="hogwild", workers=1, grid_a=8, batch_f=64),
@@ -363,7 +498,8 @@ def test_libmf_baseline_every_block_once_and_converges():
     for _ in range(20):
         g.train_epoch()
         o.train_epoch()
-        assert g.stats()["updates"] == R.N
+        assert g.stats()["updates"] == R.N           # counted by k_libmf on the device
+    assert g.check_visits()["bad_units"] == 0          # every block claimed once per epoch
     rg, ro = g.rmse(), o.rmse(R.ut, R.vt, R.rt)
     assert abs(rg - ro) <= 0.01 * ro, (rg, ro)
 
