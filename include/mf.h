@@ -124,6 +124,12 @@ typedef struct mf_params {
                              each launch is exactly what one of G GPUs runs in that sub-epoch
                              (tools/scale_emulation.py).  Same result either way: a stratum's
                              blocks touch disjoint P and Q rows                                 */
+  int32_t exact_order;    /* 1 = evaluate Alg. 1 l.8-10 in the paper's operation order, every
+                             operation rounded once (err = r - p.q; p + g((err q) - (lp p))),
+                             as the oracle does: bit-identical to it whenever the dot product is
+                             exact.  0 (default) = the fast form p' = fma(g err, q, (1-g lp) p),
+                             which rounds differently by an ulp of fp32 now and then and is
+                             8-21% faster                                 */
 } mf_params;
 
 /* Fill *p with defaults (Table 3 Netflix lambda/alpha/beta, k = 128, fp32, Hogwild, f = 256). */

@@ -800,6 +800,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->transport < 0 || p->transport > 1) return MF_E_INVAL;
   if (p->staged < 0 || p->staged > 1) return MF_E_INVAL;
   if (p->lr_rule < 0 || p->lr_rule > 1 || !(p->ada_eps >= 0.f)) return MF_E_INVAL;
+  if (p->exact_order < 0 || p->exact_order > 1) return MF_E_INVAL;
   if (p->lr_rule == 1 && p->schedule == MF_LIBMF) return MF_E_UNSUPPORTED;
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
@@ -1592,6 +1593,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     L.workers = c->p.workers; L.num_sms = c->num_sms; L.f = c->f;
     L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
     L.ada = ada_args(c);
+    L.exact = c->p.exact_order;
     if (L.ada.GP) L.g = c->p.alpha;        // ADAGRAD: constant alpha, no Eq. 9 decay
     L.out_workers = &c->last_workers; L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
     L.visits = c->visits; L.upd = c->upd_dev;
@@ -1617,6 +1619,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     L.s = c->s; L.c = c->c; L.num_sms = c->num_sms; L.P = c->P; L.Q = c->Q; L.g = g;
     L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
     L.ada = ada_args(c);
+    L.exact = c->p.exact_order;
     if (L.ada.GP) L.g = c->p.alpha;
     L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
     L.visits = c->visits + base; L.upd = c->upd_dev;
@@ -1784,6 +1787,7 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
     L.col_busy = c->lm_col; L.done = c->lm_done; L.remaining = c->lm_rem;
     L.workers = c->p.workers > 0 ? c->p.workers : std::max(1, c->a / 2);
     L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q;
+    L.exact = c->p.exact_order;
     L.seed = make_stream(c->p.seed, 11, (uint64_t)t, 0); L.stream = c->st; L.out_lanes = &c->last_lanes;
     L.visits = c->visits; L.upd = c->upd_dev;
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 0), c->st));

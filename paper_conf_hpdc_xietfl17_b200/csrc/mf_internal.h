@@ -39,6 +39,7 @@ struct HogwildLaunch {
   int workers, num_sms, f;
   void *P, *Q;
   float g, lp, lq;
+  int exact;                // params.exact_order (Step)
   AdaArgs ada;              // ada.GP != nullptr: ADAGRAD (g = alpha)
   unsigned* visits;         // per global chunk id: claims (one atomic per claimed chunk)
   unsigned long long* upd;  // non-sentinel samples updated (device count, Eq. 7)
@@ -60,6 +61,7 @@ struct WavefrontLaunch {
   int s, c, num_sms;
   void *P, *Q;
   float g, lp, lq;
+  int exact;                // params.exact_order (Step)
   AdaArgs ada;              // ada.GP != nullptr: ADAGRAD (register kernel; g = alpha)
   long long* prof;          // diagnostics (MF_PROFILE_WAVES): per worker {wait, run, samples, smid, warpid, release
                             // fence} clock64 totals, or nullptr
@@ -89,6 +91,7 @@ struct LibmfLaunch {
   int workers;
   void *P, *Q;
   float g, lp, lq;
+  int exact;                // params.exact_order (Step)
   uint64_t seed;
   unsigned* visits;         // a*a: claims of each block
   unsigned long long* upd;  // samples updated (device count)

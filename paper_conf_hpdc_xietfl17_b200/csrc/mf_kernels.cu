@@ -35,13 +35,13 @@ constexpr bool narrow16_ring(int K, int S) { return K * S == 64; }
 #ifndef MF_HOG_MINB
 #define MF_HOG_MINB 5
 #endif
-template <typename T, int K, int L, int D, bool ADA>
+template <typename T, int K, int L, int D, bool ADA, bool EX>
 __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L > 16) ? 1 : MF_HOG_MINB)
     k_hogwild(const Rating* __restrict__ slots,
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
                                                  unsigned long long* __restrict__ counter,
                                                  int workers, T* __restrict__ P, T* __restrict__ Q,
-                                                 int f, float g, float lp, float lq, AdaArgs ada,
+                                                 int f, Step st, AdaArgs ada,
                                                  unsigned* __restrict__ visits,
                                                  unsigned long long* __restrict__ upd) {
   constexpr int GPW = 32 / L;
@@ -72,7 +72,7 @@ __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L >
       if (gl == 0) atomicAdd(visits + chunk, 1u);    // exactly-once evidence (mf_check_visits)
     }
     // every group of the warp runs f iterations in lockstep (inactive ones on sentinels)
-    done += run_serial<T, K, L, D, true, ADA>(slots, lo, f, act, P, Q, g, lp, lq, gl, gbase,
+    done += run_serial<T, K, L, D, true, ADA, EX>(slots, lo, f, act, P, Q, st, gl, gbase,
                                               0xffffffffu, ada);
   }
   if (gl == 0 && done) atomicAdd(upd, (unsigned long long)done);
@@ -123,14 +123,14 @@ __device__ __forceinline__ void ticket_release(int* t, int next, unsigned gmask,
   if (gl == 0) st_relaxed(t, next);
 }
 
-template <typename T, int K, int L, bool ADA>
+template <typename T, int K, int L, bool ADA, bool EX>
 __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ slots,
                                                    const int64_t* __restrict__ sub_off,
                                                    const int32_t* __restrict__ seq,
                                                    const int32_t* __restrict__ rank,
                                                    int* __restrict__ tickets, int s, int c,
-                                                   T* __restrict__ P, T* __restrict__ Q, float g,
-                                                   float lp, float lq, int64_t shift, AdaArgs ada,
+                                                   T* __restrict__ P, T* __restrict__ Q, Step st,
+                                                   int64_t shift, AdaArgs ada,
                                                    unsigned* __restrict__ visits,
                                                    unsigned long long* __restrict__ upd) {
   const int lane = threadIdx.x & 31;
@@ -147,8 +147,8 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
     ticket_acquire(tickets + col, tgt);
     const int64_t sb = (int64_t)worker * c + col;
     const int64_t lo = __ldg(sub_off + sb) + shift;
-    done += run_serial<T, K, L, 2, false, ADA>(slots, lo, (int)(__ldg(sub_off + sb + 1) + shift - lo),
-                                               true, P, Q, g, lp, lq, gl, gbase, gmask, ada);
+    done += run_serial<T, K, L, 2, false, ADA, EX>(slots, lo, (int)(__ldg(sub_off + sb + 1) + shift - lo),
+                                               true, P, Q, st, gl, gbase, gmask, ada);
     if (gl == 0) atomicAdd(visits + sb, 1u);
     ticket_release(tickets + col, tgt + 1, gmask, gl);
   }
@@ -158,15 +158,15 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
 
 // Ring-staged wavefront (see run_subblock_ring): same schedule, tickets and result as
 // k_wavefront; the rows of each sub-block stream through a per-worker shared-memory ring.
-template <typename T, int K, int L, int RS, int F>
+template <typename T, int K, int L, int RS, int F, bool EX>
 __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ slots,
                                                     const uint16_t* __restrict__ dup,
                                                     const int64_t* __restrict__ sub_off,
                                                     const int32_t* __restrict__ seq,
                                                     const int32_t* __restrict__ rank,
                                                     int* __restrict__ tickets, int s, int c,
-                                                    T* __restrict__ P, T* __restrict__ Q, float g,
-                                                    float lp, float lq, int64_t shift,
+                                                    T* __restrict__ P, T* __restrict__ Q, Step st,
+                                                    int64_t shift,
                                                     long long* __restrict__ prof,
                                                     unsigned* __restrict__ visits,
                                                     unsigned long long* __restrict__ upd) {
@@ -216,7 +216,7 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     if (!ready) {
       ticket_acquire(tickets + col0, tgt0);   // relaxed spin + fence.acq_rel
       if (n0 > 0)
-        run_subblock_ring<T, K, L, RS, F>(slots, dup, lo0, n0, h0, P, Q, g, lp, lq, gl, gbase,
+        run_subblock_ring<T, K, L, RS, F, EX>(slots, dup, lo0, n0, h0, P, Q, st, gl, gbase,
                                           gmask, ring, true, false);
     }
     // next waves' inputs
@@ -234,13 +234,13 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     const int poll1 = w + 1 < c ? ld_acquire(tickets + col1) : -1;
     const long long tw1 = prof ? clock64() : 0;
     if (n0 > 0)
-      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo0, n0, h0, P, Q, g, lp, lq, gl, gbase, gmask,
+      run_subblock_ring<T, K, L, RS, F, EX>(slots, dup, lo0, n0, h0, P, Q, st, gl, gbase, gmask,
                                         ring, false, true);
     // next column already released: issue its row prefetch BEFORE this wave's release fence.
     // (Its p rows may have been stored by this sub-block: same thread, issued after them.)
     ready = w + 1 < c && poll1 == tgt1;
     if (ready && n1 > 0)
-      run_subblock_ring<T, K, L, RS, F>(slots, dup, lo1, n1, h1, P, Q, g, lp, lq, gl, gbase, gmask,
+      run_subblock_ring<T, K, L, RS, F, EX>(slots, dup, lo1, n1, h1, P, Q, st, gl, gbase, gmask,
                                         ring, true, false);
     const long long tw2 = prof ? clock64() : 0;
     if (gl == 0) atomicAdd(visits + (int64_t)worker * c + col0, 1u);   // sub-block (worker, col0)
@@ -281,7 +281,7 @@ __global__ void __launch_bounds__(32) k_libmf(const Rating* __restrict__ slots,
                                               const int64_t* __restrict__ blk_len, int a,
                                               int* lock, int* row_busy, int* col_busy, int* done,
                                               int* remaining, int workers, T* __restrict__ P,
-                                              T* __restrict__ Q, float g, float lp, float lq,
+                                              T* __restrict__ Q, Step st,
                                               uint64_t seed, unsigned* __restrict__ visits,
                                               unsigned long long* __restrict__ upd) {
   const int lane = threadIdx.x & 31;
@@ -333,7 +333,7 @@ __global__ void __launch_bounds__(32) k_libmf(const Rating* __restrict__ slots,
     ns = 64;
     const int64_t lo = __ldg(blk_off + b);
     if (lane == 0) atomicAdd(visits + b, 1u);
-    n_upd += run_serial<T, K, L, 1, false>(slots, lo, (int)__ldg(blk_len + b), true, P, Q, g, lp, lq,
+    n_upd += run_serial<T, K, L, 1, false>(slots, lo, (int)__ldg(blk_len + b), true, P, Q, st,
                                            lane, 0, gmask);
     __threadfence();
     __syncwarp(gmask);
@@ -436,9 +436,15 @@ cudaError_t launch_visit_check(const unsigned* visits, int64_t n, unsigned expec
 // ---------------------------------------------------------------------------------------------
 // Dispatch
 // ---------------------------------------------------------------------------------------------
-template <typename T, int K, int L, int D, bool ADA = false>
+// 1.0f and -0.0f come from here (host), opaque to the device compiler (see Step)
+template <typename Launch>
+static Step step_of(const Launch& a) {
+  return Step{a.g, a.lp, a.lq, 1.0f, -0.0f};
+}
+
+template <typename T, int K, int L, int D, bool ADA = false, bool EX = false>
 static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
-  auto kern = k_hogwild<T, K, L, D, ADA>;
+  auto kern = k_hogwild<T, K, L, D, ADA, EX>;
   const int threads = 256;
   int per_sm = 0;
   cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, 0);
@@ -452,13 +458,13 @@ static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
   if (a.out_grid) *a.out_grid = blocks;
   kern<<<blocks, threads, 0, a.stream>>>(a.slots, a.chunks, a.segs, a.counter, workers,
                                          reinterpret_cast<T*>(a.P), reinterpret_cast<T*>(a.Q), a.f,
-                                         a.g, a.lp, a.lq, a.ada, a.visits, a.upd);
+                                         step_of(a), a.ada, a.visits, a.upd);
   return cudaGetLastError();
 }
 
-template <typename T, int K, int L, bool ADA = false>
+template <typename T, int K, int L, bool ADA = false, bool EX = false>
 static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
-  auto kern = k_wavefront<T, K, L, ADA>;
+  auto kern = k_wavefront<T, K, L, ADA, EX>;
   const int threads = 128;
   const int64_t total_threads = (int64_t)a.s * L;
   const int blocks = (int)cdiv64(total_threads, threads);
@@ -476,12 +482,12 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
   int s = a.s, c = a.c;
   T* P = reinterpret_cast<T*>(a.P);
   T* Q = reinterpret_cast<T*>(a.Q);
-  float g = a.g, lp = a.lp, lq = a.lq;
+  Step st = step_of(a);
   int64_t shift = a.shift;
   AdaArgs ada = a.ada;
   unsigned* visits = a.visits;
   unsigned long long* upd = a.upd;
-  void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq, &shift,
+  void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &st, &shift,
                   &ada, &visits, &upd};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, 0,
                                      a.stream);
@@ -489,11 +495,11 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
 
 
 
-template <typename T, int K, int L, int RS_ = 0, int F_ = 0>
+template <typename T, int K, int L, int RS_ = 0, int F_ = 0, bool EX = false>
 static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
   constexpr int S = (int)sizeof(T);
   constexpr int RS = RS_ ? RS_ : ring_slots(K, S), F = F_ ? F_ : ring_ahead(K, S);
-  auto kern = k_wavefront2<T, K, L, RS, F>;
+  auto kern = k_wavefront2<T, K, L, RS, F, EX>;
   constexpr int ROWB = K * S;
   const int threads = 32;                                    // one warp = one worker
   const int wpc = 1;
@@ -516,12 +522,12 @@ static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
   int s = a.s, c = a.c;
   T* P = reinterpret_cast<T*>(a.P);
   T* Q = reinterpret_cast<T*>(a.Q);
-  float g = a.g, lp = a.lp, lq = a.lq;
+  Step st = step_of(a);
   int64_t shift = a.shift;
   long long* prof = a.prof;
   unsigned* visits = a.visits;
   unsigned long long* upd = a.upd;
-  void* args[] = {&slots, &dup, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &g, &lp, &lq,
+  void* args[] = {&slots, &dup, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &st,
                   &shift, &prof, &visits, &upd};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, smem,
                                      a.stream);
@@ -532,7 +538,7 @@ static cudaError_t launch_libmf_t(const LibmfLaunch& a) {
   if (a.out_lanes) *a.out_lanes = L;
   k_libmf<T, K, L><<<a.workers, 32, 0, a.stream>>>(
       a.slots, a.blk_off, a.blk_len, a.a, a.lock, a.row_busy, a.col_busy, a.done, a.remaining,
-      a.workers, reinterpret_cast<T*>(a.P), reinterpret_cast<T*>(a.Q), a.g, a.lp, a.lq, a.seed,
+      a.workers, reinterpret_cast<T*>(a.P), reinterpret_cast<T*>(a.Q), step_of(a), a.seed,
       a.visits, a.upd);
   return cudaGetLastError();
 }
@@ -564,6 +570,7 @@ template <typename T, int K, int LB>
 static cudaError_t hogwild_kl(const HogwildLaunch& a) {
   constexpr int S = (int)sizeof(T);
   if (a.ada.GP) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, true>(a);
+  if (a.exact) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, true>(a);  // depth 1
   if (a.prefetch == 1) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1>(a);
   return launch_hogwild_t<T, K, lanes_for(K, S, LB), 2>(a);
 }
@@ -583,25 +590,29 @@ static cudaError_t rmse_k(const RmseLaunch& a) {
   constexpr int S = (int)sizeof(T);
   return launch_rmse_t<T, K, lanes_for(K, S, 16)>(a);
 }
-template <typename T, int K>
-static cudaError_t wavefront_k(const WavefrontLaunch& a) {
+template <typename T, int K, bool EX>
+static cudaError_t wavefront_kx(const WavefrontLaunch& a) {
   constexpr int S = (int)sizeof(T);
   if (a.ada.GP) return launch_wavefront_t<T, K, lanes_for(K, S, 8), true>(a);  // register kernel
   constexpr int L2 = ring_lanes(K, S);
   constexpr int L3 = L2 / 2;                 // lane_bytes = 32: half the lanes, 32 B per lane
   if constexpr (L3 > ring_ahead(K, S) && (K * S / L3) % 16 == 0)
-    if (a.variant == 1 && a.dup && a.lane_bytes == 32) return launch_wavefront2_t<T, K, L3>(a);
+    if (a.variant == 1 && a.dup && a.lane_bytes == 32) return launch_wavefront2_t<T, K, L3, 0, 0, EX>(a);
   constexpr int L4 = L2 / 4;                 // lane_bytes = 64: a quarter of the lanes
   if constexpr (quarter_ring_ok(K, S))
-    if (a.variant == 1 && a.dup && a.lane_bytes == 64) return launch_wavefront2_t<T, K, L4, 16, 7>(a);
+    if (a.variant == 1 && a.dup && a.lane_bytes == 64) return launch_wavefront2_t<T, K, L4, 16, 7, EX>(a);
   // narrow slices on a full warp (lane_bytes = 0); lane_bytes = 16 keeps 16-B lanes
   if constexpr (narrow_ring(K, S))
-    if (a.variant == 1 && a.dup && a.lane_bytes == 0) return launch_wavefront2_t<T, K, 32, 32, 15>(a);
+    if (a.variant == 1 && a.dup && a.lane_bytes == 0) return launch_wavefront2_t<T, K, 32, 32, 15, EX>(a);
   if constexpr (narrow16_ring(K, S))
-    if (a.variant == 1 && a.dup && a.lane_bytes == 0) return launch_wavefront2_t<T, K, 16, 16, 7>(a);
+    if (a.variant == 1 && a.dup && a.lane_bytes == 0) return launch_wavefront2_t<T, K, 16, 16, 7, EX>(a);
   if constexpr (L2 > ring_ahead(K, S) && (K * S / L2) % 16 == 0)  // needs F < L, 16-B pieces
-    if (a.variant == 1 && a.dup) return launch_wavefront2_t<T, K, L2>(a);
-  return launch_wavefront_t<T, K, lanes_for(K, S, 8)>(a);
+    if (a.variant == 1 && a.dup) return launch_wavefront2_t<T, K, L2, 0, 0, EX>(a);
+  return launch_wavefront_t<T, K, lanes_for(K, S, 8), false, EX>(a);
+}
+template <typename T, int K>
+static cudaError_t wavefront_k(const WavefrontLaunch& a) {
+  return a.exact ? wavefront_kx<T, K, true>(a) : wavefront_kx<T, K, false>(a);
 }
 
 #define MF_DISPATCH(FN, ARG)                                                         \

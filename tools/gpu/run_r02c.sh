@@ -1,0 +1,3 @@
+python -m pytest tests/test_gpu_parity.py -q -p no:cacheprovider > gpurun_out/r02c_parity.log 2>&1
+python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/r02c_bench.log 2>&1
+python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --schedule wavefront --storage fp16 --workers 888 --wf-cols 7680 --cyclic > gpurun_out/r02c_wf16.log 2>&1
