@@ -6,6 +6,7 @@
 
 #include <chrono>
 #include <condition_variable>
+#include <cstdio>
 #include <cstring>
 #include <map>
 #include <memory>
@@ -26,6 +27,9 @@ struct Nccl {
   ncclResult_t (*GroupStart)() = nullptr;
   ncclResult_t (*GroupEnd)() = nullptr;
   const char* (*ErrStr)(ncclResult_t) = nullptr;
+  ncclResult_t (*CommCount)(const ncclComm_t, int*) = nullptr;      // optional (logging)
+  ncclResult_t (*CommCuDevice)(const ncclComm_t, int*) = nullptr;   // optional (logging)
+  ncclResult_t (*GetVersion)(int*) = nullptr;                       // optional (logging)
 };
 
 Nccl* nccl(std::string* why) {
@@ -49,6 +53,9 @@ Nccl* nccl(std::string* why) {
     SYM(GroupStart, "ncclGroupStart");
     SYM(GroupEnd, "ncclGroupEnd");
     SYM(ErrStr, "ncclGetErrorString");
+    SYM(CommCount, "ncclCommCount");
+    SYM(CommCuDevice, "ncclCommCuDevice");
+    SYM(GetVersion, "ncclGetVersion");
 #undef SYM
     ok = lib.CommInitRank && lib.CommDestroy && lib.Send && lib.Recv && lib.Bcast &&
          lib.AllReduce && lib.GroupStart && lib.GroupEnd && lib.ErrStr;
@@ -165,6 +172,19 @@ Comm* Comm::create(const uint8_t id[128], int world, int rank, cudaStream_t st, 
   std::memcpy(&uid, id, 128);
   ncclComm_t cm = nullptr;
   if (!check(L, L->CommInitRank(&cm, world, uid, rank), "ncclCommInitRank", why)) return nullptr;
+  // one line per rank on stderr: the communicator really spans `world` ranks (the driver's
+  // multi-GPU record checks the count)
+  int nranks = -1, dev = -1, ver = 0;
+  if (L->CommCount) L->CommCount(cm, &nranks);
+  if (L->CommCuDevice) L->CommCuDevice(cm, &dev);
+  if (L->GetVersion) L->GetVersion(&ver);
+  std::fprintf(stderr, "[mf_comm] NCCL communicator ready: rank %d of %d, ncclCommCount = %d, "
+                       "cuda device %d, NCCL %d\n", rank, world, nranks, dev, ver);
+  if (L->CommCount && nranks != world) {
+    L->CommDestroy(cm);
+    if (why) *why = "ncclCommCount differs from world";
+    return nullptr;
+  }
   Comm* c = new Comm();
   c->comm_ = cm;
   c->st_ = st;

@@ -49,3 +49,24 @@ def test_bench_reference_arm_line():
     assert d["impl"] == "reference" and d["value"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle"
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["d2h_bytes_per_step"] == 0
+
+
+@pytest.mark.parametrize("ranks", [2, 4])
+def test_bench_multirank_path_emulated(ranks):
+    """bench.py's N > 1 code path (Hugewiki-shaped DSGD strata, configs[3]) with N ranks as
+    threads on one GPU over the library's loopback transport: the JSON line of N GPUs with its
+    e2e (out-of-core epochs, H2D counted over all ranks), cpu_baseline, exactly-once record and
+    the device-counted updates adding up to N per epoch -- so the first real multi-GPU run
+    cannot die on a bench bug."""
+    d = _bench("--emulate-ranks", str(ranks), "--steps", "3", "--warmup", "3", "--fraction", "0.002",
+               "--e2e-steps", "1", "--cpu-sample", "20000")
+    assert d["n_gpus"] == ranks and d["scaling"] == "strong"
+    assert d["config"]["workload"].startswith("hugewiki") and d["config"]["grid_a"] == 8
+    assert d["config"]["parallelism"] == f"dsgd-strata{ranks}"
+    eo = d["exactly_once"]
+    assert eo["bad_units"] == 0 and eo["updates_per_epoch"] == eo["N"] == d["config"]["N_train"]
+    assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0
+    assert d["e2e"]["d2h_bytes_per_step"] == 8 * ranks
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["gpu_launches"] > 0
+    assert d["emulated_ranks"]["ranks"] == ranks
+    assert d["test_rmse"] < d["test_rmse_init"]
