@@ -54,6 +54,8 @@ def parse():
     ap.add_argument("--lane-bytes", type=int, default=0)
     ap.add_argument("--prefetch", type=int, default=0)
     ap.add_argument("--wf-kernel", type=int, default=0)
+    ap.add_argument("--rating-stage", type=int, default=0,
+                    help="Hogwild rating stream: 0 = per-lane loads, 1 = TMA bulk copies")
     ap.add_argument("--exact-order", action="store_true",
                     help="evaluate Alg. 1 l.8-10 in the paper's operation order (params.exact_order)")
     ap.add_argument("--staged", action="store_true",
@@ -320,6 +322,7 @@ def config_of(args, R, world):
             "storage": args.storage, "schedule": args.schedule, "batch_f": default_f(args, world),
             "parallelism": f"dsgd-strata{world}" if world > 1 else "1gpu",
             "fraction": args.fraction, "exact_order": bool(args.exact_order),
+            "rating_stage": "tma" if args.rating_stage else "lane-loads",
             "staged": bool(args.staged), "grid_a": args.grid_a or (8 if world > 1 else 1),
             "l2": "inputs larger than L2 (COO %.2f GB per epoch); model P+Q stays cached as in "
                   "any training run" % (R.N * 12 / 1e9)}
@@ -354,7 +357,7 @@ def rank_main(args, C, R=None, out=None):
               wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes,
               prefetch=args.prefetch, wf_kernel=args.wf_kernel, grid_a=args.grid_a,
               batch_f=default_f(args, world), lr_rule=args.lr_rule, seed=42,
-              exact_order=args.exact_order, device=C.local, rank=rank, world=world,
+              exact_order=args.exact_order, rating_stage=args.rating_stage, device=C.local, rank=rank, world=world,
               nccl_id=nccl_id, transport=C.transport, **hp)
     torch.cuda.synchronize()
     model = mf.MF(R.m, R.n, args.k, stream=stream, staged=args.staged, **kw)
@@ -404,7 +407,8 @@ def rank_main(args, C, R=None, out=None):
     traffic, tsrc = ncu_traffic(args) if world == 1 else (None, None)
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
             "frac": achieved / hbm, "traffic": traffic, "peak_source": peak_src,
-            "kernel": f"k_{args.schedule}", "bytes_per_update": bpu,
+            "kernel": f"k_{args.schedule}", "bytes_per_update": bpu, "workers": st["workers"],
+            "lanes_per_worker": st["lanes"], "grid": st["grid"],
             "sgd_ms_per_epoch": float(np.mean(sgd_ms)), "sched_ms_per_epoch": float(np.mean(sched_ms)),
             "step_achieved": value / world * bpu / 1e9, "step_frac": value / world * bpu / 1e9 / hbm}
     if traffic:

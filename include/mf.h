@@ -130,6 +130,11 @@ typedef struct mf_params {
                              exact.  0 (default) = the fast form p' = fma(g err, q, (1-g lp) p),
                              which rounds differently by an ulp of fp32 now and then and is
                              8-21% faster                                 */
+  int32_t rating_stage;   /* Hogwild rating stream (north_star (2), Eq. 8 batches): 0 = per-lane
+                             streaming loads + warp shuffles; 1 = TMA: one lane per worker
+                             bulk-copies its chunk into shared memory in 768-B sub-chunks
+                             (cp.async.bulk + mbarrier, double buffered).  1 needs f % 64 == 0,
+                             prefetch 1 and the default 16-B lanes (else MF_E_UNSUPPORTED)    */
 } mf_params;
 
 /* Fill *p with defaults (Table 3 Netflix lambda/alpha/beta, k = 128, fp32, Hogwild, f = 256). */

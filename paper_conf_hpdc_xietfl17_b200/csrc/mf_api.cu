@@ -801,6 +801,10 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->staged < 0 || p->staged > 1) return MF_E_INVAL;
   if (p->lr_rule < 0 || p->lr_rule > 1 || !(p->ada_eps >= 0.f)) return MF_E_INVAL;
   if (p->exact_order < 0 || p->exact_order > 1) return MF_E_INVAL;
+  if (p->rating_stage < 0 || p->rating_stage > 1) return MF_E_INVAL;
+  if (p->rating_stage == 1 && ((p->batch_f > 0 ? p->batch_f : 256) % 64 != 0 ||
+                               p->prefetch > 1 || (p->lane_bytes && p->lane_bytes != 16)))
+    return MF_E_UNSUPPORTED;                      // TMA stream: f % 64 == 0, default geometry
   if (p->lr_rule == 1 && p->schedule == MF_LIBMF) return MF_E_UNSUPPORTED;
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
@@ -1589,6 +1593,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     HogwildLaunch L{};
     L.storage = c->p.storage; L.k = c->k; L.lane_bytes = c->p.lane_bytes ? c->p.lane_bytes : 16;
     L.prefetch = c->p.prefetch ? c->p.prefetch : 1;
+    L.rating_stage = c->p.rating_stage;
     L.slots = slots; L.chunks = c->chunk_order; L.segs = segs; L.counter = c->counter;
     L.workers = c->p.workers; L.num_sms = c->num_sms; L.f = c->f;
     L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;

@@ -35,7 +35,7 @@ constexpr bool narrow16_ring(int K, int S) { return K * S == 64; }
 #ifndef MF_HOG_MINB
 #define MF_HOG_MINB 5
 #endif
-template <typename T, int K, int L, int D, bool ADA, bool EX>
+template <typename T, int K, int L, int D, bool ADA, bool EX, int SRC>
 __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L > 16) ? 1 : MF_HOG_MINB)
     k_hogwild(const Rating* __restrict__ slots,
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
@@ -53,6 +53,22 @@ __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L >
   const int nact = min(GPW, workers - first);
   const int64_t total = segs.prefix[segs.n];
   int done = 0;                                      // this group's non-sentinel updates
+  // SRC = 1: this group's rating ring in dynamic shared memory (2 mbarriers + 2 x 768 B)
+  extern __shared__ __align__(16) char hsm[];
+  RatingRing ring{};
+  unsigned phase = 0;
+  if constexpr (SRC == 1) {
+    const int gid = (int)(threadIdx.x >> 5) * GPW + grp;   // group within the CTA
+    const int ngroups = (int)(blockDim.x >> 5) * GPW;
+    ring.bar = reinterpret_cast<uint64_t*>(hsm) + 2 * gid;
+    ring.buf = hsm + 16 * ngroups + 2 * kSubBytes * gid;
+    if (gl == 0) {
+      mbar_init(ring.bar, 1);
+      mbar_init(ring.bar + 1, 1);
+      mbar_init_fence();
+    }
+    __syncwarp();
+  }
   for (;;) {
     unsigned long long base = 0;
     if (lane == 0) base = atomicAdd(counter, (unsigned long long)nact);
@@ -72,8 +88,8 @@ __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L >
       if (gl == 0) atomicAdd(visits + chunk, 1u);    // exactly-once evidence (mf_check_visits)
     }
     // every group of the warp runs f iterations in lockstep (inactive ones on sentinels)
-    done += run_serial<T, K, L, D, true, ADA, EX>(slots, lo, f, act, P, Q, st, gl, gbase,
-                                              0xffffffffu, ada);
+    done += run_serial<T, K, L, D, true, ADA, EX, SRC>(slots, lo, f, act, P, Q, st, gl, gbase,
+                                                       0xffffffffu, ada, ring, &phase);
   }
   if (gl == 0 && done) atomicAdd(upd, (unsigned long long)done);
 }
@@ -442,12 +458,24 @@ static Step step_of(const Launch& a) {
   return Step{a.g, a.lp, a.lq, 1.0f, -0.0f};
 }
 
-template <typename T, int K, int L, int D, bool ADA = false, bool EX = false>
+template <typename T, int K, int L, int D, bool ADA = false, bool EX = false, int SRC = 0>
 static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
-  auto kern = k_hogwild<T, K, L, D, ADA, EX>;
+  auto kern = k_hogwild<T, K, L, D, ADA, EX, SRC>;
   const int threads = 256;
+  const int groups = threads / 32 * (32 / L);
+  const size_t smem = SRC == 1 ? (size_t)groups * (16 + 2 * kSubBytes) : 0;
+  cudaError_t e;
+  if (SRC == 1) {
+    if (a.f % kSub != 0) return cudaErrorInvalidValue;     // mf_create rejects it first
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    // the rings need the shared-memory carveout that keeps MF_HOG_MINB blocks resident
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout,
+                             cudaSharedmemCarveoutMaxShared);
+    if (e != cudaSuccess) return e;
+  }
   int per_sm = 0;
-  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, 0);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, smem);
   if (e != cudaSuccess) return e;
   const int gpw = 32 / L;
   const int resident_workers = per_sm * a.num_sms * (threads / 32) * gpw;
@@ -456,7 +484,7 @@ static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
   if (a.out_workers) *a.out_workers = workers;
   if (a.out_lanes) *a.out_lanes = L;
   if (a.out_grid) *a.out_grid = blocks;
-  kern<<<blocks, threads, 0, a.stream>>>(a.slots, a.chunks, a.segs, a.counter, workers,
+  kern<<<blocks, threads, smem, a.stream>>>(a.slots, a.chunks, a.segs, a.counter, workers,
                                          reinterpret_cast<T*>(a.P), reinterpret_cast<T*>(a.Q), a.f,
                                          step_of(a), a.ada, a.visits, a.upd);
   return cudaGetLastError();
@@ -571,6 +599,8 @@ static cudaError_t hogwild_kl(const HogwildLaunch& a) {
   constexpr int S = (int)sizeof(T);
   if (a.ada.GP) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, true>(a);
   if (a.exact) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, true>(a);  // depth 1
+  if (a.rating_stage == 1 && LB == 16)
+    return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, false, 1>(a);        // TMA stream
   if (a.prefetch == 1) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1>(a);
   return launch_hogwild_t<T, K, lanes_for(K, S, LB), 2>(a);
 }

@@ -54,7 +54,8 @@ class Params(ctypes.Structure):
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
                 ("transport", ctypes.c_int32), ("nccl_id", ctypes.c_void_p),
                 ("stream", ctypes.c_void_p), ("alloc", ctypes.POINTER(Allocator)),
-                ("launch_blocks", ctypes.c_int32), ("exact_order", ctypes.c_int32)]
+                ("launch_blocks", ctypes.c_int32), ("exact_order", ctypes.c_int32),
+                ("rating_stage", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -189,7 +190,7 @@ class MF:
                  batch_f: int = 256, wf_cols: int = 0, grid_a: int = 0, cyclic: bool = False,
                  lane_bytes: int = 0, prefetch: int = 0, wf_kernel: int = 0, staged: bool = False,
                  lr_rule: str = "eq9", ada_eps: float = 1e-8, launch_blocks: int = 0,
-                 exact_order: bool = False,
+                 exact_order: bool = False, rating_stage: int = 0,
                  device: int = 0, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, transport: int = 0, stream=None,
                  allocator: str = "torch"):
@@ -207,6 +208,7 @@ class MF:
         p.staged = int(staged)
         p.launch_blocks = launch_blocks
         p.exact_order = int(exact_order)
+        p.rating_stage = int(rating_stage)
         p.lr_rule, p.ada_eps = {"eq9": 0, "adagrad": 1}[lr_rule], ada_eps
         p.device, p.rank, p.world, p.transport = device, rank, world, transport
         self._id_buf = None

@@ -311,6 +311,46 @@ def test_appendix_a_hand_pins_through_the_abi(golden_dir):
     assert t.export("perm").tolist() == g0["perm_S_SHUF_10"]
 
 
+@pytest.mark.parametrize("kw", [dict(k=128, storage="fp16"), dict(k=128, storage="fp32"),
+                                dict(k=32, storage="fp16"), dict(k=256, storage="bf16"),
+                                dict(k=64, storage="fp32", grid_a=4, batch_f=128),
+                                dict(k=128, storage="fp16", grid_a=4, batch_f=64, staged=True)])
+def test_tma_rating_stream_equals_register_stream(kw):
+    """rating_stage = 1 (the chunk's ratings bulk-copied into shared memory by the TMA engine,
+    768-B sub-chunks, mbarrier-tracked, double buffered) feeds the same samples in the same
+    order as the per-lane load + shuffle stream: 1-worker runs are bit-identical, and both
+    match the oracle (fp32: 1e-4); at full concurrency every chunk is claimed once."""
+    kw = dict(kw)
+    k = kw.pop("k")
+    R = ragged()
+    out = []
+    for stage in (0, 1):
+        g = mf.MF(R.m, R.n, k, workers=1, rating_stage=stage, **TABLE3_NETFLIX, **kw)
+        g.load(R.u, R.v, R.r)
+        g.load(R.ut, R.vt, R.rt, "test")
+        for _ in range(2):
+            g.train_epoch()
+        assert g.stats()["updates"] == R.N
+        out.append((g.factors(), g.rmse()))
+        g.close()
+    (P0, Q0), r0 = out[0]
+    (P1, Q1), r1 = out[1]
+    assert np.array_equal(P0, P1) and np.array_equal(Q0, Q1) and r0 == r1
+    if kw["storage"] == "fp32":
+        o = po.Oracle(R.m, R.n, k, R.u, R.v, R.r, **TABLE3_NETFLIX,
+                      **{kk: vv for kk, vv in kw.items() if kk != "staged"})
+        o.train_epoch()
+        o.train_epoch()
+        Po, Qo = o.factors()
+        assert np.abs(P1 - Po).max() <= 1e-4 and np.abs(Q1 - Qo).max() <= 1e-4
+    g = mf.MF(R.m, R.n, k, rating_stage=1, **TABLE3_NETFLIX, **kw)    # all resident workers
+    g.load(R.u, R.v, R.r)
+    for _ in range(3):
+        g.train_epoch()
+        assert g.stats()["updates"] == R.N
+    assert g.check_visits()["bad_units"] == 0
+
+
 def test_hogwild_one_worker_reproduces_oracle_curve(tiny):
     """1 worker = the serial batch-Hogwild order of the oracle: the RMSE curve matches epoch by
     epoch -- 1e-5 relative after epoch 1 (north_star), and within 1e-4 over 10 epochs as the

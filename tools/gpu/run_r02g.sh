@@ -1,0 +1,7 @@
+python -m pytest tests/test_gpu_parity.py -q -p no:cacheprovider -k "tma or staged or exactly_once" > gpurun_out/r02g_tests.log 2>&1
+for st in 0 1; do
+python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --no-deterministic --rating-stage $st > gpurun_out/r02g_netflix_rs$st.log 2>&1
+python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --no-deterministic --rating-stage $st --workload yahoo > gpurun_out/r02g_yahoo_rs$st.log 2>&1
+python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --no-deterministic --rating-stage $st --storage fp32 > gpurun_out/r02g_netflix32_rs$st.log 2>&1
+python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-e2e --no-deterministic --rating-stage $st --k 32 > gpurun_out/r02g_netflixk32_rs$st.log 2>&1
+done
