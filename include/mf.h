@@ -100,8 +100,10 @@ typedef struct mf_params {
                              G += g^2, step alpha*g/sqrt(G + ada_eps); Hogwild and register
                              wavefront kernels                                                  */
   float ada_eps;          /* ADAGRAD epsilon (0 = 1e-8)                                         */
-  int32_t staged;         /* 1 = out-of-core ratings (section 6.2): after the GPU
-                             preprocessing the bucketed ratings live in pinned host memory and
+  int32_t staged;         /* 1 = out-of-core ratings (section 6.2): the bucketed
+                             ratings live in pinned host memory (a host train set is
+                             preprocessed in chunks of stage_chunk samples, never whole in
+                             HBM; a device set is preprocessed resident, then moved) and
                              each stratum's blocks stream into one of two HBM buffers on a copy
                              stream while the previous stratum computes; P, Q stay resident.
                              When n <= 65535 the host copy and the H2D stream carry 10-B
@@ -135,6 +137,10 @@ typedef struct mf_params {
                              bulk-copies its chunk into shared memory in 768-B sub-chunks
                              (cp.async.bulk + mbarrier, double buffered).  1 needs f % 64 == 0,
                              prefetch 1 and the default 16-B lanes (else MF_E_UNSUPPORTED)    */
+  int64_t stage_chunk;    /* staged = 1 with a HOST train set: samples per chunk of the
+                             out-of-core preprocessing (0 = 2^26).  Device memory then holds one
+                             chunk (~68 B per sample) or one strata block (~60 B per sample) at a
+                             time instead of the whole set (section 6)            */
 } mf_params;
 
 /* Fill *p with defaults (Table 3 Netflix lambda/alpha/beta, k = 128, fp32, Hogwild, f = 256). */

@@ -447,6 +447,61 @@ float gamma_of(float alpha, float beta, int32_t t) {
   return (float)((double)alpha / (1.0 + (double)beta * td * std::sqrt(td)));
 }
 
+// ---- out-of-core (chunked) preprocessing (section 6): the caller's COO streams
+// through the device in chunks; pass 1 partitions each chunk by strata block, pass 2 orders one
+// block at a time.  Same slots as the resident path, bit for bit.
+// Pass 1: record i0 + j of the caller's set -> (block, shuffle key, relabelled rating).  Samples
+// of row segments this rank does not own get block = nb (sorted last, dropped).
+__global__ void k_chunk_records(const int32_t* __restrict__ u, const int32_t* __restrict__ v,
+                                const float* __restrict__ r, int64_t C, int64_t i0, uint64_t S,
+                                const int32_t* __restrict__ rho_r, const int32_t* __restrict__ rho_c,
+                                double rs, int64_t m, int64_t n, int64_t a, int64_t lo_seg,
+                                int64_t hi_seg, uint32_t* __restrict__ blk,
+                                uint32_t* __restrict__ idx, uint64_t* __restrict__ keys,
+                                Rating* __restrict__ recs) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < C;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    Rating x;
+    x.u = rho_r[u[j]];
+    x.v = rho_c[v[j]];
+    x.r = (float)((double)r[j] / rs);                  // R5, rounded once (as k_build_storage)
+    const int64_t seg = (int64_t)x.u * a / m;
+    const bool own = seg >= lo_seg && seg < hi_seg;
+    blk[j] = own ? (uint32_t)(seg * a + (int64_t)x.v * a / n) : (uint32_t)(a * a);
+    idx[j] = (uint32_t)j;
+    keys[j] = hkey(S, (uint64_t)(i0 + j));              // A: key(S_SHUF, caller index)
+    recs[j] = x;
+  }
+}
+
+__global__ void k_iota_u32(uint32_t* __restrict__ x, int64_t n) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n;
+       j += (int64_t)gridDim.x * blockDim.x)
+    x[j] = (uint32_t)j;
+}
+
+__global__ void k_gather_records(const uint32_t* __restrict__ order, int64_t n,
+                                 const uint64_t* __restrict__ kin, const Rating* __restrict__ rin,
+                                 uint64_t* __restrict__ kout, Rating* __restrict__ rout) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t o = order[j];
+    if (kout) kout[j] = kin[o];
+    rout[j] = rin[o];
+  }
+}
+
+// Pass 2 (wavefront): sub-block of each (key-ordered) sample of block b, local to the block.
+__global__ void k_local_sub(const Rating* __restrict__ recs, int64_t n, Grid G, int64_t b,
+                            uint32_t* __restrict__ sub, uint32_t* __restrict__ idx) {
+  const int64_t per = G.s * G.c;
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    sub[j] = (uint32_t)((int64_t)bucket_of(G, recs[j].u, recs[j].v) - b * per);
+    idx[j] = (uint32_t)j;
+  }
+}
+
 // A: host perm of a small set (strata order pi_t).
 std::vector<int64_t> host_perm(uint64_t S, int64_t n) {
   std::vector<std::pair<uint64_t, int64_t>> t((size_t)n);
@@ -1030,9 +1085,8 @@ static mf_status alloc_schedule(mf_ctx* c) {
   return MF_OK;
 }
 
-// Move the bucketed ratings (and the wavefront dup metadata) to pinned host memory and size
-// the two device staging buffers for the largest stratum this rank can meet:
-// sum over owned row segments r of max_J |block (r, J)|.
+// Move the bucketed ratings (and the wavefront dup metadata) from HBM to pinned host memory
+// (the resident preprocessing path; the chunked path writes them there directly).
 static mf_status setup_staging(mf_ctx* c) {
   CUDA_TRY(c, cudaStreamSynchronize(c->st));
   const size_t ns = (size_t)std::max<int64_t>(c->nslots, 1);
@@ -1071,6 +1125,12 @@ static mf_status setup_staging(mf_ctx* c) {
   c->release(c->dup);
   c->release(c->slot_pos);
   c->release(c->perm);
+  return MF_OK;
+}
+
+// The two device staging buffers, sized for the largest stratum this rank can meet:
+// sum over owned row segments r of max_J |block (r, J)|; the copy stream and its events.
+static mf_status setup_staging_buffers(mf_ctx* c) {
   int64_t cap = 1;
   int64_t sum = 0;
   for (int r = c->lo_row_seg(); r < c->hi_row_seg(); ++r) {
@@ -1339,7 +1399,255 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
   TRY(c->alloc(&c->visits, (size_t)std::max<int64_t>(c->n_units, 1)));
   CUDA_TRY(c, cudaMemsetAsync(c->visits, 0, (size_t)std::max<int64_t>(c->n_units, 1) * 4, c->st));
   c->epochs_run = 0;
-  if (c->staged) TRY(setup_staging(c));
+  if (c->staged) {
+    TRY(setup_staging(c));
+    TRY(setup_staging_buffers(c));
+  }
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  c->train_loaded = true;
+  return MF_OK;
+}
+
+
+// ---------------------------------------------------------------------------------------------
+// Out-of-core load (params.staged with a HOST rating set; section 6, "partition the
+// data sets and stage the partitions to GPUs in batches"): the caller's COO never resides in
+// HBM as a whole.  Device memory holds one chunk of stage_chunk samples (pass 1) or one strata
+// block (pass 2) at a time, so a set larger than the device budget loads.
+//   pass 1, per chunk: H2D, validate, relabel, strata block + shuffle key key(S_SHUF, i) of
+//     every sample (i = caller index, 64-bit), stable sort by block, D2H appended to per-block
+//     host runs (rank-foreign samples dropped);
+//   pass 2, per block: H2D its runs, sort by key (= the storage order of Alg. 1 l.2 restricted
+//     to the block, R12), wavefront: stable sort by sub-block, sub-block offsets and duplicate
+//     distances; padded (Hogwild) and written to the pinned host slots the epochs stream from.
+// The slots are those of the resident path, bit for bit (tests/test_gpu_parity.py), and
+// N >= 2^32 is allowed (keys and block runs are 64-bit indexed; a block must stay < 2^32).
+// ---------------------------------------------------------------------------------------------
+static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, const int32_t* v,
+                                    const float* r) {
+  const int64_t nb = (int64_t)c->a * c->a;
+  const int64_t C = std::max<int64_t>(
+      1, std::min<int64_t>(std::max<int64_t>(N, 1),
+                           c->p.stage_chunk > 0 ? c->p.stage_chunk : ((int64_t)1 << 26)));
+  TRY(relabel(c, kTagRow, c->m, &c->rho_r));
+  TRY(relabel(c, kTagCol, c->n, &c->rho_c));
+  const uint64_t S = make_stream(c->p.seed, kTagShuf, 0, 0);
+  std::vector<std::vector<uint64_t>> hk((size_t)nb);
+  std::vector<std::vector<Rating>> hr((size_t)nb);
+  std::vector<int64_t> bcount((size_t)nb, 0);
+  {  // ---- pass 1
+    int32_t *cu = nullptr, *cv = nullptr;
+    float* cr = nullptr;
+    uint32_t *b0 = nullptr, *b1 = nullptr, *i0 = nullptr, *i1 = nullptr;
+    uint64_t *k0 = nullptr, *k1 = nullptr;
+    Rating *r0 = nullptr, *r1 = nullptr;
+    int* bad = nullptr;
+    unsigned* cnt = nullptr;
+    TRY(c->alloc(&cu, (size_t)C)); TRY(c->alloc(&cv, (size_t)C)); TRY(c->alloc(&cr, (size_t)C));
+    TRY(c->alloc(&b0, (size_t)C)); TRY(c->alloc(&b1, (size_t)C));
+    TRY(c->alloc(&i0, (size_t)C)); TRY(c->alloc(&i1, (size_t)C));
+    TRY(c->alloc(&k0, (size_t)C)); TRY(c->alloc(&k1, (size_t)C));
+    TRY(c->alloc(&r0, (size_t)C)); TRY(c->alloc(&r1, (size_t)C));
+    TRY(c->alloc(&bad, 1)); TRY(c->alloc(&cnt, (size_t)nb + 1));
+    uint64_t* hkb = nullptr;
+    Rating* hrb = nullptr;
+    CUDA_TRY(c, cudaMallocHost(&hkb, (size_t)C * 8));
+    CUDA_TRY(c, cudaMallocHost(&hrb, (size_t)C * sizeof(Rating)));
+    std::vector<unsigned> hc((size_t)nb + 1);
+    mf_status st = MF_OK;
+    for (int64_t s0 = 0; s0 < N && st == MF_OK; s0 += C) {
+      const int64_t n = std::min(C, N - s0);
+      const int g = grid_for(n, c->num_sms);
+      cudaError_t e = cudaMemcpyAsync(cu, u + s0, (size_t)n * 4, cudaMemcpyHostToDevice, c->st);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(cv, v + s0, (size_t)n * 4, cudaMemcpyHostToDevice, c->st);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(cr, r + s0, (size_t)n * 4, cudaMemcpyHostToDevice, c->st);
+      if (e == cudaSuccess) e = cudaMemsetAsync(bad, 0, 4, c->st);
+      if (e != cudaSuccess) { st = c->cuda_fail(e, "chunk H2D", __LINE__); break; }
+      k_validate<<<g, 256, 0, c->st>>>(cu, cv, cr, n, c->m, c->n, bad);
+      int hbad = 0;
+      e = cudaMemcpyAsync(&hbad, bad, 4, cudaMemcpyDeviceToHost, c->st);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(c->st);
+      if (e != cudaSuccess) { st = c->cuda_fail(e, "chunk validate", __LINE__); break; }
+      if (hbad) { st = c->fail(MF_E_RANGE, "rating index out of range or non-finite rating"); break; }
+      k_chunk_records<<<g, 256, 0, c->st>>>(cu, cv, cr, n, s0, S, c->rho_r, c->rho_c,
+                                            (double)c->p.rating_scale, c->m, c->n, c->a,
+                                            c->lo_row_seg(), c->hi_row_seg(), b0, i0, k0, r0);
+      if ((e = cudaGetLastError()) != cudaSuccess) { st = c->cuda_fail(e, "k_chunk_records", __LINE__); break; }
+      if ((st = c->sort_pairs(b0, b1, i0, i1, n, bits_for((uint64_t)nb))) != MF_OK) break;
+      k_gather_records<<<g, 256, 0, c->st>>>(i1, n, k0, r0, k1, r1);
+      e = cudaMemsetAsync(cnt, 0, (nb + 1) * 4, c->st);
+      if (nb + 1 <= kSmemBuckets)
+        k_histogram_smem<<<g, 256, 0, c->st>>>(b1, n, (int)nb + 1, cnt);
+      else
+        k_histogram<<<g, 256, 0, c->st>>>(b1, n, cnt);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(hc.data(), cnt, (nb + 1) * 4, cudaMemcpyDeviceToHost, c->st);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(hkb, k1, (size_t)n * 8, cudaMemcpyDeviceToHost, c->st);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(hrb, r1, (size_t)n * sizeof(Rating), cudaMemcpyDeviceToHost, c->st);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(c->st);
+      if (e != cudaSuccess) { st = c->cuda_fail(e, "chunk partition", __LINE__); break; }
+      int64_t off = 0;                       // the chunk's block runs, in block order
+      for (int64_t b = 0; b < nb; ++b) {
+        const int64_t len = hc[(size_t)b];
+        if (len) {
+          hk[(size_t)b].insert(hk[(size_t)b].end(), hkb + off, hkb + off + len);
+          hr[(size_t)b].insert(hr[(size_t)b].end(), hrb + off, hrb + off + len);
+        }
+        bcount[(size_t)b] += len;
+        off += len;
+      }
+    }
+    cudaFreeHost(hkb);
+    cudaFreeHost(hrb);
+    for (void* x : {(void*)cu, (void*)cv, (void*)cr, (void*)b0, (void*)b1, (void*)i0, (void*)i1,
+                    (void*)k0, (void*)k1, (void*)r0, (void*)r1, (void*)bad, (void*)cnt}) {
+      void* y = x;
+      c->release(y);
+    }
+    if (st != MF_OK) return st;
+  }
+  // ---- block layout (A: padding of Hogwild blocks to a multiple of f)
+  int64_t Nown = 0, maxlen = 1;
+  c->blk_off.assign((size_t)nb + 1, 0);
+  c->blk_len.assign((size_t)nb, 0);
+  c->ch_off.assign((size_t)nb + 1, 0);
+  for (int64_t b = 0; b < nb; ++b) {
+    const int64_t len = bcount[(size_t)b];
+    if (len >= ((int64_t)1 << 32)) return c->fail(MF_E_UNSUPPORTED, "a strata block holds >= 2^32 ratings");
+    Nown += len;
+    c->blk_len[(size_t)b] = len;
+    const int64_t padded = c->wf ? len : cdiv64(len, c->f) * c->f;
+    c->ch_off[(size_t)b + 1] = c->ch_off[(size_t)b] + (c->wf ? 0 : cdiv64(len, c->f));
+    c->blk_off[(size_t)b + 1] = c->blk_off[(size_t)b] + padded;
+    maxlen = std::max(maxlen, padded);
+  }
+  c->N = Nown;
+  c->nslots = c->blk_off.back();
+  const size_t ns = (size_t)std::max<int64_t>(c->nslots, 1);
+  c->stg_packed = c->n <= 65535;
+  if (c->stg_packed) {
+    CUDA_TRY(c, cudaMallocHost(&c->h_u, ns * 4));
+    CUDA_TRY(c, cudaMallocHost(&c->h_v16, ns * 2));
+    CUDA_TRY(c, cudaMallocHost(&c->h_r, ns * 4));
+  } else {
+    CUDA_TRY(c, cudaMallocHost(&c->h_slots, ns * sizeof(Rating)));
+  }
+  const bool want_dup = c->wf && c->p.wf_kernel != 2;
+  if (want_dup) CUDA_TRY(c, cudaMallocHost(&c->h_dup, ns * sizeof(uint16_t)));
+  // ---- pass 2
+  {
+    Grid Gd{c->m, c->n, c->a, c->s, c->c, c->wf};
+    const int64_t per = (int64_t)c->s * c->c;
+    uint64_t *k0 = nullptr, *k1 = nullptr;
+    uint32_t *i0 = nullptr, *i1 = nullptr, *s0 = nullptr, *s1 = nullptr;
+    Rating *r0 = nullptr, *r1 = nullptr;
+    unsigned* cnt = nullptr;
+    uint16_t* dd = nullptr;
+    int32_t* du = nullptr;
+    uint16_t* dv = nullptr;
+    float* dr = nullptr;
+    TRY(c->alloc(&k0, (size_t)maxlen)); TRY(c->alloc(&k1, (size_t)maxlen));
+    TRY(c->alloc(&i0, (size_t)maxlen)); TRY(c->alloc(&i1, (size_t)maxlen));
+    TRY(c->alloc(&r0, (size_t)maxlen)); TRY(c->alloc(&r1, (size_t)maxlen));
+    if (c->wf) {
+      TRY(c->alloc(&s0, (size_t)maxlen)); TRY(c->alloc(&s1, (size_t)maxlen));
+      TRY(c->alloc(&cnt, (size_t)per));
+    }
+    if (want_dup) TRY(c->alloc(&dd, (size_t)maxlen));
+    if (c->stg_packed) {
+      TRY(c->alloc(&du, (size_t)maxlen)); TRY(c->alloc(&dv, (size_t)maxlen));
+      TRY(c->alloc(&dr, (size_t)maxlen));
+    }
+    std::vector<int64_t> subo;
+    std::vector<unsigned> hcnt;
+    if (c->wf) {
+      subo.assign((size_t)(nb * per + 1), 0);
+      hcnt.resize((size_t)per);
+    }
+    const int W = want_dup ? ring_window(c->k, c->p.storage, c->p.lane_bytes) : 0;
+    for (int64_t b = 0; b < nb; ++b) {
+      const int64_t len = c->blk_len[(size_t)b], lo = c->blk_off[(size_t)b];
+      const int64_t padded = c->blk_off[(size_t)b + 1] - lo;
+      if (c->wf)
+        for (int64_t q = 0; q <= per; ++q) subo[(size_t)(b * per + q)] = lo;   // empty default
+      if (len == 0) continue;
+      const int g = grid_for(len, c->num_sms);
+      CUDA_TRY(c, cudaMemcpyAsync(k0, hk[(size_t)b].data(), (size_t)len * 8, cudaMemcpyHostToDevice, c->st));
+      CUDA_TRY(c, cudaMemcpyAsync(r0, hr[(size_t)b].data(), (size_t)len * sizeof(Rating),
+                                  cudaMemcpyHostToDevice, c->st));
+      k_iota_u32<<<g, 256, 0, c->st>>>(i0, len);
+      KERNEL_TRY(c);
+      TRY(c->sort_pairs(k0, k1, i0, i1, len, 64));                 // storage order in the block
+      k_gather_records<<<g, 256, 0, c->st>>>(i1, len, nullptr, r0, nullptr, r1);
+      KERNEL_TRY(c);
+      Rating* fin = r1;
+      if (c->wf) {
+        k_local_sub<<<g, 256, 0, c->st>>>(r1, len, Gd, b, s0, i0);
+        KERNEL_TRY(c);
+        TRY(c->sort_pairs(s0, s1, i0, i1, len, bits_for((uint64_t)std::max<int64_t>(per - 1, 1))));
+        k_gather_records<<<g, 256, 0, c->st>>>(i1, len, nullptr, r1, nullptr, r0);
+        CUDA_TRY(c, cudaMemsetAsync(cnt, 0, (size_t)per * 4, c->st));
+        k_histogram<<<g, 256, 0, c->st>>>(s1, len, cnt);
+        KERNEL_TRY(c);
+        CUDA_TRY(c, cudaMemcpyAsync(hcnt.data(), cnt, (size_t)per * 4, cudaMemcpyDeviceToHost, c->st));
+        fin = r0;
+        if (want_dup) {
+          k_dupdist<<<g, 256, 0, c->st>>>(fin, len, Gd, W, dd);
+          KERNEL_TRY(c);
+          CUDA_TRY(c, cudaMemcpyAsync(c->h_dup + lo, dd, (size_t)len * 2, cudaMemcpyDeviceToHost, c->st));
+        }
+      } else if (padded > len) {
+        CUDA_TRY(c, cudaMemsetAsync(fin + len, 0xFF, (size_t)(padded - len) * sizeof(Rating), c->st));
+      }
+      if (c->stg_packed) {
+        k_split_slots<<<grid_for(padded, c->num_sms), 256, 0, c->st>>>(fin, padded, du, dv, dr);
+        KERNEL_TRY(c);
+        CUDA_TRY(c, cudaMemcpyAsync(c->h_u + lo, du, (size_t)padded * 4, cudaMemcpyDeviceToHost, c->st));
+        CUDA_TRY(c, cudaMemcpyAsync(c->h_v16 + lo, dv, (size_t)padded * 2, cudaMemcpyDeviceToHost, c->st));
+        CUDA_TRY(c, cudaMemcpyAsync(c->h_r + lo, dr, (size_t)padded * 4, cudaMemcpyDeviceToHost, c->st));
+      } else {
+        CUDA_TRY(c, cudaMemcpyAsync(c->h_slots + lo, fin, (size_t)padded * sizeof(Rating),
+                                    cudaMemcpyDeviceToHost, c->st));
+      }
+      CUDA_TRY(c, cudaStreamSynchronize(c->st));
+      if (c->wf) {
+        int64_t run = lo;
+        for (int64_t q = 0; q < per; ++q) {
+          subo[(size_t)(b * per + q)] = run;
+          run += hcnt[(size_t)q];
+        }
+        subo[(size_t)(b * per + per)] = run;
+      }
+      std::vector<uint64_t>().swap(hk[(size_t)b]);               // host runs of b done
+      std::vector<Rating>().swap(hr[(size_t)b]);
+    }
+    for (void* x : {(void*)k0, (void*)k1, (void*)i0, (void*)i1, (void*)r0, (void*)r1, (void*)s0,
+                    (void*)s1, (void*)cnt, (void*)dd, (void*)du, (void*)dv, (void*)dr}) {
+      void* y = x;
+      c->release(y);
+    }
+    if (c->wf) {
+      TRY(c->alloc(&c->sub_off, subo.size()));
+      CUDA_TRY(c, cudaMemcpyAsync(c->sub_off, subo.data(), subo.size() * 8, cudaMemcpyHostToDevice, c->st));
+      CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    } else {
+      TRY(c->alloc(&c->d_choff, (size_t)nb + 1));
+      CUDA_TRY(c, cudaMemcpyAsync(c->d_choff, c->ch_off.data(), (nb + 1) * 8, cudaMemcpyHostToDevice, c->st));
+      CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    }
+  }
+  TRY(init_factors(c));
+  if (c->p.lr_rule == 1) {
+    TRY(c->alloc(&c->GP, (size_t)(c->m * c->k)));
+    TRY(c->alloc(&c->GQ, (size_t)(c->n * c->k)));
+    CUDA_TRY(c, cudaMemsetAsync(c->GP, 0, (size_t)(c->m * c->k) * 4, c->st));
+    CUDA_TRY(c, cudaMemsetAsync(c->GQ, 0, (size_t)(c->n * c->k) * 4, c->st));
+  }
+  TRY(alloc_schedule(c));
+  c->n_units = c->wf ? nb * (int64_t)c->s * c->c : c->ch_off.back();
+  TRY(c->alloc(&c->visits, (size_t)std::max<int64_t>(c->n_units, 1)));
+  CUDA_TRY(c, cudaMemsetAsync(c->visits, 0, (size_t)std::max<int64_t>(c->n_units, 1) * 4, c->st));
+  c->epochs_run = 0;
+  TRY(setup_staging_buffers(c));
   CUDA_TRY(c, cudaStreamSynchronize(c->st));
   c->train_loaded = true;
   return MF_OK;
@@ -1404,7 +1712,9 @@ mf_status mf_load_coo(mf_ctx* c, int32_t set, int64_t nnz, const int32_t* u, con
   mf_status s = MF_OK;
   if (set == MF_TRAIN) {
     if (c->train_loaded) return c->fail(MF_E_STATE, "train set already loaded");
-    s = load_train(c, nnz, u, v, r, on_device);
+    // out-of-core mode with a host rating set: chunked preprocessing (never all in HBM)
+    s = (c->staged && !on_device) ? load_train_chunked(c, nnz, u, v, r)
+                                  : load_train(c, nnz, u, v, r, on_device);
   } else if (set == MF_TEST) {
     if (!c->train_loaded) return c->fail(MF_E_STATE, "load the train set first");
     if (c->test_loaded) return c->fail(MF_E_STATE, "test set already loaded");

@@ -55,7 +55,7 @@ class Params(ctypes.Structure):
                 ("transport", ctypes.c_int32), ("nccl_id", ctypes.c_void_p),
                 ("stream", ctypes.c_void_p), ("alloc", ctypes.POINTER(Allocator)),
                 ("launch_blocks", ctypes.c_int32), ("exact_order", ctypes.c_int32),
-                ("rating_stage", ctypes.c_int32)]
+                ("rating_stage", ctypes.c_int32), ("stage_chunk", ctypes.c_int64)]
 
 
 class Stats(ctypes.Structure):
@@ -145,22 +145,32 @@ def _torch():
 
 
 class _TorchAllocator:
-    """mf_allocator hooks backed by torch's CUDA caching allocator."""
+    """mf_allocator hooks backed by torch's CUDA caching allocator.  `budget` (bytes, optional)
+    caps the ctx's live device memory: an allocation beyond it returns NULL (MF_E_NOMEM), the
+    way a device smaller than the problem would; `peak` records the high-water mark."""
 
-    def __init__(self, device: int):
+    def __init__(self, device: int, budget: int | None = None):
         torch = _torch()
         self.device = device
         self.sizes = {}
+        self.live = 0
+        self.peak = 0
 
         def _alloc(nbytes, stream, user):
+            if budget is not None and self.live + int(nbytes) > budget:
+                return None
             try:
                 ptr = torch.cuda.caching_allocator_alloc(int(nbytes), device, int(stream or 0))
-                return ptr
             except Exception:  # OOM -> NULL -> MF_E_NOMEM
                 return None
+            self.sizes[ptr] = int(nbytes)
+            self.live += int(nbytes)
+            self.peak = max(self.peak, self.live)
+            return ptr
 
         def _free(ptr, nbytes, stream, user):
             if ptr:
+                self.live -= self.sizes.pop(ptr, 0)
                 torch.cuda.caching_allocator_delete(ptr)
 
         self._a = _ALLOC_FN(_alloc)
@@ -190,10 +200,10 @@ class MF:
                  batch_f: int = 256, wf_cols: int = 0, grid_a: int = 0, cyclic: bool = False,
                  lane_bytes: int = 0, prefetch: int = 0, wf_kernel: int = 0, staged: bool = False,
                  lr_rule: str = "eq9", ada_eps: float = 1e-8, launch_blocks: int = 0,
-                 exact_order: bool = False, rating_stage: int = 0,
+                 exact_order: bool = False, rating_stage: int = 0, stage_chunk: int = 0,
                  device: int = 0, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, transport: int = 0, stream=None,
-                 allocator: str = "torch"):
+                 allocator: str = "torch", device_budget: int | None = None):
         L = lib()
         p = Params()
         L.mf_params_default(ctypes.byref(p))
@@ -209,6 +219,7 @@ class MF:
         p.launch_blocks = launch_blocks
         p.exact_order = int(exact_order)
         p.rating_stage = int(rating_stage)
+        p.stage_chunk = int(stage_chunk)
         p.lr_rule, p.ada_eps = {"eq9": 0, "adagrad": 1}[lr_rule], ada_eps
         p.device, p.rank, p.world, p.transport = device, rank, world, transport
         self._id_buf = None
@@ -222,7 +233,7 @@ class MF:
             p.stream = ctypes.c_void_p(int(getattr(stream, "cuda_stream", stream)) or None)
         self._alloc = None
         if allocator == "torch" and torch.cuda.is_available():
-            self._alloc = _TorchAllocator(device)
+            self._alloc = _TorchAllocator(device, device_budget)
             p.alloc = ctypes.pointer(self._alloc.struct)
         self.params = p
         self.m, self.n, self.k = int(m), int(n), int(k)
@@ -330,6 +341,11 @@ class MF:
         self._check(lib().mf_check_visits(self.h, ctypes.byref(bad), ctypes.byref(units),
                                           ctypes.byref(ep)), "mf_check_visits")
         return {"bad_units": bad.value, "units": units.value, "epochs": ep.value}
+
+    @property
+    def device_peak_bytes(self) -> int:
+        """High-water mark of the ctx's device memory (torch allocator hooks only)."""
+        return self._alloc.peak if self._alloc is not None else -1
 
     def stats(self) -> dict:
         s = Stats()

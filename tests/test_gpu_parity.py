@@ -489,6 +489,47 @@ def test_checkpoint_resume_equals_uninterrupted(tiny):
 
 # ----------------------------------------------------------------------------- out-of-core
 
+@pytest.mark.parametrize("kw", [dict(schedule="hogwild", workers=1, grid_a=8, batch_f=64),
+                                dict(schedule="wavefront", workers=4, wf_cols=6, grid_a=8),
+                                dict(schedule="hogwild", workers=1, grid_a=8, batch_f=256,
+                                     storage="fp16")])
+def test_out_of_core_load_below_the_device_budget_is_bit_identical(kw):
+    """Section 6: a rating set larger than the device memory it may use.  The ctx
+    gets a device budget BELOW the 12-B COO of its training set (the torch allocator hook refuses
+    anything beyond it, as a smaller device would); the staged load streams the host set through
+    chunked preprocessing and the epochs stream it from pinned host memory.  The trained model is
+    bit-identical to the resident run (deterministic schedules: wavefront, 1-worker Hogwild),
+    and every sample is updated exactly once per epoch."""
+    R = synth.uniform(m=5000, n=2000, N=2_000_000, seed=3, mu=0.5, rank=4, noise=0.1, Ntest=5000)
+    coo = 12 * R.N
+    out = []
+    for staged in (False, True):
+        extra = dict(staged=True, stage_chunk=1 << 17, device_budget=coo * 3 // 4) if staged else {}
+        g = mf.MF(R.m, R.n, 32, **TABLE3_NETFLIX, **kw, **extra)
+        g.load(R.u, R.v, R.r)                       # host arrays
+        g.load(R.ut, R.vt, R.rt, "test")
+        g.train_epoch()
+        assert g.stats()["updates"] == R.N
+        assert g.check_visits()["bad_units"] == 0
+        if staged:
+            assert 0 < g.device_peak_bytes < coo, (g.device_peak_bytes, coo)
+        out.append((g.factors(), g.rmse()))
+        g.close()
+    (P0, Q0), r0 = out[0]
+    (P1, Q1), r1 = out[1]
+    assert np.array_equal(P0, P1) and np.array_equal(Q0, Q1) and r0 == r1
+
+
+def test_resident_load_fails_cleanly_below_the_device_budget():
+    """The same budget without out-of-core staging: the resident preprocessing needs the whole
+    set in HBM, so the load fails with MF_E_NOMEM (and the ctx stays usable)."""
+    R = synth.uniform(m=5000, n=2000, N=2_000_000, seed=3, mu=0.5, rank=4, noise=0.1)
+    g = mf.MF(R.m, R.n, 32, grid_a=8, device_budget=12 * R.N * 3 // 4)
+    with pytest.raises(mf.MFError) as e:
+        g.load(R.u, R.v, R.r)
+    assert e.value.status == -2
+
+
 @pytest.mark.parametrize("staged", [False, True])
 def test_destroy_right_after_an_epoch_with_the_default_allocator(staged):
     """an epoch in staged mode ends by queueing the next stratum's H2D copy on the
