@@ -56,6 +56,8 @@ def parse():
     ap.add_argument("--wf-kernel", type=int, default=0)
     ap.add_argument("--rating-stage", type=int, default=0,
                     help="Hogwild rating stream: 0 = per-lane loads, 1 = TMA bulk copies")
+    ap.add_argument("--group-cols", action="store_true",
+                    help="batch-Hogwild with column-grouped batches (reading R24, params.group_cols)")
     ap.add_argument("--exact-order", action="store_true",
                     help="evaluate Alg. 1 l.8-10 in the paper's operation order (params.exact_order)")
     ap.add_argument("--staged", action="store_true",
@@ -323,6 +325,7 @@ def config_of(args, R, world):
             "parallelism": f"dsgd-strata{world}" if world > 1 else "1gpu",
             "fraction": args.fraction, "exact_order": bool(args.exact_order),
             "rating_stage": "tma" if args.rating_stage else "lane-loads",
+            "group_cols": bool(args.group_cols),
             "staged": bool(args.staged), "grid_a": args.grid_a or (8 if world > 1 else 1),
             "l2": "inputs larger than L2 (COO %.2f GB per epoch); model P+Q stays cached as in "
                   "any training run" % (R.N * 12 / 1e9)}
@@ -357,7 +360,8 @@ def rank_main(args, C, R=None, out=None):
               wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes,
               prefetch=args.prefetch, wf_kernel=args.wf_kernel, grid_a=args.grid_a,
               batch_f=default_f(args, world), lr_rule=args.lr_rule, seed=42,
-              exact_order=args.exact_order, rating_stage=args.rating_stage, device=C.local, rank=rank, world=world,
+              exact_order=args.exact_order, rating_stage=args.rating_stage,
+              group_cols=args.group_cols, device=C.local, rank=rank, world=world,
               nccl_id=nccl_id, transport=C.transport, **hp)
     torch.cuda.synchronize()
     model = mf.MF(R.m, R.n, args.k, stream=stream, staged=args.staged, **kw)

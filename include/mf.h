@@ -141,6 +141,13 @@ typedef struct mf_params {
                              out-of-core preprocessing (0 = 2^26).  Device memory then holds one
                              chunk (~68 B per sample) or one strata block (~60 B per sample) at a
                              time instead of the whole set (section 6)            */
+  int32_t group_cols;     /* batch-Hogwild, reading R24: every batch of f consecutive samples
+                             (Eq. 8; "fetch f consecutive samples and update them serially",
+                             P:L272) is updated in order of (relabelled column, storage
+                             position) instead of storage order, so repeated -- power-law-hot --
+                             columns of a batch run back to back and their q_v stays in
+                             registers (no load, no intermediate store).  The oracle runs the
+                             same order (or_params.group_cols).  Hogwild only                */
 } mf_params;
 
 /* Fill *p with defaults (Table 3 Netflix lambda/alpha/beta, k = 128, fp32, Hogwild, f = 256). */

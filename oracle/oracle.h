@@ -64,6 +64,8 @@ typedef struct or_params {
   int32_t cyclic;          /* wavefront cyclic column order variant (A: cyclic) */
   int32_t lr_rule;         /* 0 = Eq. 9 schedule; 1 = ADAGRAD (or_update_adagrad, R23) */
   float   ada_eps;         /* ADAGRAD epsilon */
+  int32_t group_cols;      /* batch-Hogwild, reading R24: inside each batch of f consecutive
+                              samples, update them in order of (relabelled column, position) */
 } or_params;
 
 typedef struct or_ctx or_ctx;

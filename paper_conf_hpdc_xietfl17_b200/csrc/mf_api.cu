@@ -474,6 +474,27 @@ __global__ void k_chunk_records(const int32_t* __restrict__ u, const int32_t* __
   }
 }
 
+// Column-grouped batches (group_cols, reading R24): key of slot x of a chunk-aligned piece =
+// (chunk within the piece, relabelled column); a stable sort by it orders every batch of f
+// consecutive samples by column, ties in storage order (sentinel pads, v = -1, stay last).
+__global__ void k_group_keys(const Rating* __restrict__ slots, int64_t n, int f,
+                             uint64_t* __restrict__ keys, uint32_t* __restrict__ vals) {
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    keys[x] = ((uint64_t)(x / f) << 32) | (uint32_t)slots[x].v;
+    vals[x] = (uint32_t)x;
+  }
+}
+__global__ void k_permute_slots(const uint32_t* __restrict__ order, int64_t n,
+                                const Rating* __restrict__ in, Rating* __restrict__ out,
+                                const uint32_t* __restrict__ pin, uint32_t* __restrict__ pout) {
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    out[x] = in[order[x]];
+    if (pout) pout[x] = pin[order[x]];
+  }
+}
+
 __global__ void k_iota_u32(uint32_t* __restrict__ x, int64_t n) {
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n;
        j += (int64_t)gridDim.x * blockDim.x)
@@ -856,6 +877,9 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->staged < 0 || p->staged > 1) return MF_E_INVAL;
   if (p->lr_rule < 0 || p->lr_rule > 1 || !(p->ada_eps >= 0.f)) return MF_E_INVAL;
   if (p->exact_order < 0 || p->exact_order > 1) return MF_E_INVAL;
+  if (p->group_cols < 0 || p->group_cols > 1) return MF_E_INVAL;
+  if (p->group_cols && (p->schedule != MF_HOGWILD || p->rating_stage || p->prefetch > 1))
+    return MF_E_UNSUPPORTED;
   if (p->rating_stage < 0 || p->rating_stage > 1) return MF_E_INVAL;
   if (p->rating_stage == 1 && ((p->batch_f > 0 ? p->batch_f : 256) % 64 != 0 ||
                                p->prefetch > 1 || (p->lane_bytes && p->lane_bytes != 16)))
@@ -1202,6 +1226,35 @@ static mf_status stage(mf_ctx* c, int32_t t, int32_t j, int buf) {
   return MF_OK;
 }
 
+// group_cols (R24): order every Hogwild batch of f slots in [lo, lo + len) (a padded strata
+// block, chunk aligned) by column, in pieces of at most ~2^26 slots (whole chunks).
+static mf_status group_batches(mf_ctx* c, Rating* slots, uint32_t* slot_pos, int64_t len) {
+  if (!c->p.group_cols || len == 0) return MF_OK;
+  const int64_t piece = std::max<int64_t>(c->f, (((int64_t)1 << 26) / c->f) * c->f);
+  const int64_t cap = std::min(piece, len);
+  uint64_t *k0 = nullptr, *k1 = nullptr;
+  uint32_t *v0 = nullptr, *v1 = nullptr, *p1 = nullptr;
+  Rating* tmp = nullptr;
+  TRY(c->alloc(&k0, (size_t)cap)); TRY(c->alloc(&k1, (size_t)cap));
+  TRY(c->alloc(&v0, (size_t)cap)); TRY(c->alloc(&v1, (size_t)cap));
+  TRY(c->alloc(&tmp, (size_t)cap));
+  if (slot_pos) TRY(c->alloc(&p1, (size_t)cap));
+  for (int64_t lo = 0; lo < len; lo += piece) {
+    const int64_t n = std::min(piece, len - lo);
+    const int g = grid_for(n, c->num_sms);
+    k_group_keys<<<g, 256, 0, c->st>>>(slots + lo, n, c->f, k0, v0);
+    KERNEL_TRY(c);
+    TRY(c->sort_pairs(k0, k1, v0, v1, n, 32 + bits_for((uint64_t)cdiv64(n, c->f))));
+    k_permute_slots<<<g, 256, 0, c->st>>>(v1, n, slots + lo, tmp, slot_pos ? slot_pos + lo : nullptr, p1);
+    KERNEL_TRY(c);
+    CUDA_TRY(c, cudaMemcpyAsync(slots + lo, tmp, (size_t)n * sizeof(Rating), cudaMemcpyDeviceToDevice, c->st));
+    if (slot_pos)
+      CUDA_TRY(c, cudaMemcpyAsync(slot_pos + lo, p1, (size_t)n * 4, cudaMemcpyDeviceToDevice, c->st));
+  }
+  c->release(k0); c->release(k1); c->release(v0); c->release(v1); c->release(tmp); c->release(p1);
+  return MF_OK;
+}
+
 static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_t* v,
                             const float* r, int on_device) {
   if (N >= (int64_t)UINT32_MAX) return c->fail(MF_E_UNSUPPORTED, "N >= 2^32 not supported");
@@ -1378,6 +1431,11 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
   if (!c->wf) { c->release(src_off); c->release(dst_off); }
   c->release(cnt); c->release(stor); c->release(bk0); c->release(bk1);
   c->release(pos0); c->release(pos1);
+  if (!c->wf && !c->libmf)
+    for (int64_t b = 0; b < nb; ++b)
+      TRY(group_batches(c, c->slots + c->blk_off[(size_t)b],
+                        c->slot_pos ? c->slot_pos + c->blk_off[(size_t)b] : nullptr,
+                        c->blk_off[(size_t)b + 1] - c->blk_off[(size_t)b]));
 
   if (c->wf && c->p.wf_kernel != 2) {
     TRY(c->alloc(&c->dup, (size_t)std::max<int64_t>(c->nslots, 1)));
@@ -1595,8 +1653,10 @@ static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, cons
           KERNEL_TRY(c);
           CUDA_TRY(c, cudaMemcpyAsync(c->h_dup + lo, dd, (size_t)len * 2, cudaMemcpyDeviceToHost, c->st));
         }
-      } else if (padded > len) {
-        CUDA_TRY(c, cudaMemsetAsync(fin + len, 0xFF, (size_t)(padded - len) * sizeof(Rating), c->st));
+      } else {
+        if (padded > len)
+          CUDA_TRY(c, cudaMemsetAsync(fin + len, 0xFF, (size_t)(padded - len) * sizeof(Rating), c->st));
+        TRY(group_batches(c, fin, nullptr, padded));
       }
       if (c->stg_packed) {
         k_split_slots<<<grid_for(padded, c->num_sms), 256, 0, c->st>>>(fin, padded, du, dv, dr);
@@ -1904,6 +1964,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     L.storage = c->p.storage; L.k = c->k; L.lane_bytes = c->p.lane_bytes ? c->p.lane_bytes : 16;
     L.prefetch = c->p.prefetch ? c->p.prefetch : 1;
     L.rating_stage = c->p.rating_stage;
+    L.group = c->p.group_cols;
     L.slots = slots; L.chunks = c->chunk_order; L.segs = segs; L.counter = c->counter;
     L.workers = c->p.workers; L.num_sms = c->num_sms; L.f = c->f;
     L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;

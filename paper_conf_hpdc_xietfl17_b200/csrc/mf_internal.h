@@ -33,6 +33,7 @@ struct ChunkSegs {
 struct HogwildLaunch {
   int storage, k, lane_bytes, prefetch;
   int rating_stage;         // 0 = per-lane streaming loads + shuffles, 1 = TMA bulk copies
+  int group;                // params.group_cols: column-grouped batches (R24)
   const Rating* slots;
   const uint32_t* chunks;
   ChunkSegs segs;

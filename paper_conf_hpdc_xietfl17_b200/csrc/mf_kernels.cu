@@ -35,7 +35,7 @@ constexpr bool narrow16_ring(int K, int S) { return K * S == 64; }
 #ifndef MF_HOG_MINB
 #define MF_HOG_MINB 5
 #endif
-template <typename T, int K, int L, int D, bool ADA, bool EX, int SRC>
+template <typename T, int K, int L, int D, bool ADA, bool EX, int SRC, bool GRP>
 __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L > 16) ? 1 : MF_HOG_MINB)
     k_hogwild(const Rating* __restrict__ slots,
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
@@ -88,7 +88,7 @@ __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L >
       if (gl == 0) atomicAdd(visits + chunk, 1u);    // exactly-once evidence (mf_check_visits)
     }
     // every group of the warp runs f iterations in lockstep (inactive ones on sentinels)
-    done += run_serial<T, K, L, D, true, ADA, EX, SRC>(slots, lo, f, act, P, Q, st, gl, gbase,
+    done += run_serial<T, K, L, D, true, ADA, EX, SRC, GRP>(slots, lo, f, act, P, Q, st, gl, gbase,
                                                        0xffffffffu, ada, ring, &phase);
   }
   if (gl == 0 && done) atomicAdd(upd, (unsigned long long)done);
@@ -458,9 +458,10 @@ static Step step_of(const Launch& a) {
   return Step{a.g, a.lp, a.lq, 1.0f, -0.0f};
 }
 
-template <typename T, int K, int L, int D, bool ADA = false, bool EX = false, int SRC = 0>
+template <typename T, int K, int L, int D, bool ADA = false, bool EX = false, int SRC = 0,
+          bool GRP = false>
 static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
-  auto kern = k_hogwild<T, K, L, D, ADA, EX, SRC>;
+  auto kern = k_hogwild<T, K, L, D, ADA, EX, SRC, GRP>;
   const int threads = 256;
   const int groups = threads / 32 * (32 / L);
   const size_t smem = SRC == 1 ? (size_t)groups * (16 + 2 * kSubBytes) : 0;
@@ -597,6 +598,11 @@ static constexpr int lanes_for(int K, int S, int LB) {
 template <typename T, int K, int LB>
 static cudaError_t hogwild_kl(const HogwildLaunch& a) {
   constexpr int S = (int)sizeof(T);
+  if (a.group) {                                 // column-grouped batches (R24), depth 1
+    if (a.ada.GP) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, true, false, 0, true>(a);
+    if (a.exact) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, true, 0, true>(a);
+    return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, false, 0, true>(a);
+  }
   if (a.ada.GP) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, true>(a);
   if (a.exact) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, true>(a);  // depth 1
   if (a.rating_stage == 1 && LB == 16)

@@ -578,3 +578,44 @@ def test_adagrad_training_converges_on_tiny():
         losses.append(o.loss())
     assert o.rmse(R.ut, R.vt, R.rt) < 0.5 * r0
     assert losses[-1] < 0.2 * losses[0]
+
+
+# --------------------------------------------------------------------------- R24 grouped batches
+
+def test_grouped_batches_order_hand_derived(golden_dir):
+    """Reading R24: inside every batch of f consecutive samples the order is (relabelled
+    column, storage position); the batch order itself is unchanged (A: S_HW)."""
+    g = golden(golden_dir, "grouped_batches.json")
+    cs = g["case"]
+    u = np.array(cs["u"], np.int32)
+    v = np.array(cs["v"], np.int32)
+    r = np.ones(len(u), np.float32)
+    o = po.Oracle(cs["m"], cs["n"], 16, u, v, r, seed=42, batch_f=cs["f"], group_cols=True)
+    assert o.export("perm").tolist() == g["perm_S_SHUF_10"]
+    assert o.export("rho_c").tolist() == g["rho_C"]
+    assert o.export("chunkorder", 0).tolist() == g["chunk_order_t0"]
+    assert o.export("order", 0).tolist() == g["order_grouped_t0"]
+    plain = po.Oracle(cs["m"], cs["n"], 16, u, v, r, seed=42, batch_f=cs["f"])
+    assert plain.export("order", 0).tolist() == g["order_plain_t0"]
+
+
+def test_grouped_batches_permute_within_batches_only():
+    """Property at any size: the grouped order is the plain order with each batch's samples
+    permuted among themselves (same batches, same batch order, each sample once), and within a
+    batch the relabelled columns are non-decreasing."""
+    u, v, r, m, n = _tiny_uniform(m=97, n=13, N=4000)
+    f = 64
+    og = po.Oracle(m, n, 4, u, v, r, group_cols=True, seed=3, batch_f=f)
+    op = po.Oracle(m, n, 4, u, v, r, seed=3, batch_f=f)
+    a, b = og.export("order", 1), op.export("order", 1)
+    assert sorted(a.tolist()) == list(range(4000))
+    perm, rho_c = og.export("perm"), og.export("rho_c")
+    pos = 0
+    for q in og.export("chunkorder", 1):                  # one strata block: list = storage order
+        batch = list(range(q * f, min(q * f + f, 4000)))
+        assert b[pos:pos + len(batch)].tolist() == batch
+        seg = a[pos:pos + len(batch)]
+        assert sorted(seg.tolist()) == batch
+        assert np.all(np.diff(rho_c[v[perm[seg]]]) >= 0)
+        pos += len(batch)
+    assert pos == 4000
