@@ -430,9 +430,11 @@ def rank_main(args, C, R=None, out=None):
     e2e = None
     if not args.no_e2e and not (big and world == 1):
         e2e = run_e2e(args, R, kw, stream, C)
-    det = None
+    det = grp = None
     if not args.no_deterministic and world == 1 and args.schedule == "hogwild" and not big:
         det = run_deterministic(args, R, hp, stream)
+        if not args.group_cols:
+            grp = run_grouped(args, R, hp, stream)
     cpu = None
     if not args.no_cpu_baseline and rank == 0:
         cpu = cpu_baseline(R, hp, args, args.cpu_sample)
@@ -452,7 +454,7 @@ def rank_main(args, C, R=None, out=None):
             "exactly_once": {"bad_units": int(bad_units), "units": visits["units"],
                              "epochs": visits["epochs"], "updates_per_epoch": all_updates / args.steps,
                              "N": R.N},
-            "e2e": e2e, "cpu_baseline": cpu, "deterministic": det,
+            "e2e": e2e, "cpu_baseline": cpu, "deterministic": det, "grouped": grp,
             "paper_context": "cuMF_SGD Table 5 (P:L414-415), fp16 Hogwild: Netflix 267M/s TITAN X, "
                              "613M/s P100; Hugewiki 256M/s / 710M/s (other hardware; context only)"}
     if isinstance(C, ThreadRank):
@@ -502,6 +504,43 @@ def run_deterministic(args, R, hp, stream):
            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                         "frac": achieved / hbm, "bytes_per_update": bpu,
                         "step_frac": upd / (ms / 1000.0) * bpu / 1e9 / hbm}}
+    m.close()
+    return out
+
+
+def run_grouped(args, R, hp, stream):
+    """The same Hogwild run with column-grouped batches (reading R24, params.group_cols) at
+    f = 1024 (profiles/r02_grouped_batches.md): device-timed like the main line, same data."""
+    from paper_conf_hpdc_xietfl17_b200 import mf
+    steps, warm = max(3, args.steps // 2), 3
+    m = mf.MF(R.m, R.n, args.k, stream=stream, schedule="hogwild", storage=args.storage,
+              group_cols=True, batch_f=1024, seed=42, **hp)
+    m.load(R.u, R.v, R.r, "train")
+    m.load(R.ut, R.vt, R.rt, "test")
+    for _ in range(warm):
+        m.train_epoch()
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    sgd, upd = [], 0
+    e0.record(stream)
+    for _ in range(steps):
+        m.train_epoch()
+        st = m.stats()
+        sgd.append(st["sgd_ms"])
+        upd += st["updates"]
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    hbm, _ = peaks()
+    bpu = st["bytes_per_update"]
+    achieved = upd * bpu / (float(np.sum(sgd)) / 1000.0) / 1e9
+    out = {"schedule": "hogwild, column-grouped batches (R24), f=1024", "storage": args.storage,
+           "value": upd / (ms / 1000.0), "unit": "updates/s", "ms_per_step": ms / steps,
+           "steps": steps, "warmup": warm, "test_rmse": m.rmse("test"),
+           "exactly_once_bad_units": m.check_visits()["bad_units"],
+           "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                        "frac": achieved / hbm, "bytes_per_update": bpu}}
     m.close()
     return out
 

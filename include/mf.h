@@ -148,6 +148,12 @@ typedef struct mf_params {
                              columns of a batch run back to back and their q_v stays in
                              registers (no load, no intermediate store).  The oracle runs the
                              same order (or_params.group_cols).  Hogwild only                */
+  int32_t check_owners;   /* debug (deterministic wavefront): tag each column block with its
+                             holder on acquire (atomicCAS) and check the tag on release; any
+                             overlap of two holders is counted (mf_owner_violations) -- the
+                             mutual exclusion of the ticket protocol on the global P/Q rows,
+                             which compute-sanitizer's racecheck (shared memory only) cannot
+                             see.  One atomic per wave when on, nothing when off             */
 } mf_params;
 
 /* Fill *p with defaults (Table 3 Netflix lambda/alpha/beta, k = 128, fp32, Hogwild, f = 256). */
@@ -180,6 +186,12 @@ mf_status mf_train_epoch(mf_ctx* ctx, int32_t* epoch_done);
  * fp64 accumulation, deterministic reduction order.  world > 1: global value (all ranks).
  * Synchronises.  MF_E_RANGE if the result is NaN (divergence). */
 mf_status mf_rmse(mf_ctx* ctx, int32_t set, double* out);
+
+/* Eq. 2 over the training set: sum over train ratings of (r' - p_u.q_v)^2 +
+ * lambda_p ||p_u||^2 + lambda_q ||q_v||^2, in the scaled rating units r' = r / rating_scale the
+ * model trains on; fp32 dots and norms per sample, fp64 accumulation.  world > 1: the global
+ * value on every rank.  Resident ratings only (MF_E_UNSUPPORTED when staged).  Synchronises. */
+mf_status mf_loss(mf_ctx* ctx, double* out);
 
 /* Copy the model out in ORIGINAL ids as fp32 (Alg. 1 l.15 model_shuffle): P is m x k
  * row-major, Q is n x k row-major (row v = q_v, R14).  Either pointer may be NULL.
@@ -236,6 +248,10 @@ mf_status mf_get_stats(mf_ctx* ctx, mf_stats* out);
  * this rank does not train) and writes the number of mismatching units to *bad_units, the
  * number of units to *units and the epochs to *epochs (either may be NULL).  Synchronises. */
 mf_status mf_check_visits(mf_ctx* ctx, int64_t* bad_units, int64_t* units, int32_t* epochs);
+
+/* Ownership-checker violations counted since load (params.check_owners = 1, wavefront;
+ * MF_E_STATE otherwise).  0 = no two workers ever held a column block at the same time. */
+mf_status mf_owner_violations(mf_ctx* ctx, int64_t* violations);
 
 /* Per-launch device times (ms, CUDA events) of the SGD launches of the last epoch, in launch
  * order (synchronises).  With ms == NULL only *n is set; otherwise *n must be >= the count and

@@ -13,6 +13,7 @@
 #include <cstdlib>
 #include <map>
 #include <cub/cub.cuh>
+#include <nvtx3/nvToolsExt.h>
 #include <string>
 #include <vector>
 
@@ -21,6 +22,22 @@
 #include "mf_internal.h"
 
 using namespace mfb;
+
+// NVTX ranges (SURVEY 5 tracing): per load phase, epoch, schedule build, sub-epoch, Q rotation
+// and evaluation -- visible in nsys / ncu --nvtx timelines; header-only, no cost unattached.
+struct Nvtx {
+  explicit Nvtx(const char* fmt, ...) {
+    char buf[96];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    nvtxRangePushA(buf);
+  }
+  ~Nvtx() { nvtxRangePop(); }
+  Nvtx(const Nvtx&) = delete;
+  Nvtx& operator=(const Nvtx&) = delete;
+};
 
 // =============================================================================================
 // preprocessing / schedule kernels
@@ -591,6 +608,8 @@ struct mf_ctx {
   unsigned long long* upd_dev = nullptr;
   unsigned long long* chk_dev = nullptr;
   int32_t epochs_run = 0;
+  int* owners = nullptr;             // params.check_owners: wavefront column tags (c)
+  unsigned* own_viol = nullptr;      // violations found by the ownership checker
   double* rm_partial = nullptr;
   double* rm_out = nullptr;
   void* tmp = nullptr;
@@ -739,7 +758,8 @@ struct mf_ctx {
         (void**)&d_blk_len, (void**)&lm_lock, (void**)&lm_row, (void**)&lm_col, (void**)&lm_done,
         (void**)&lm_rem, (void**)&stg[0], (void**)&stg[1], (void**)&stg_dup[0],
         (void**)&stg_dup[1], (void**)&stg_u[0], (void**)&stg_u[1], (void**)&stg_v16[0],
-        (void**)&stg_v16[1], (void**)&stg_r[0], (void**)&stg_r[1], (void**)&visits};
+        (void**)&stg_v16[1], (void**)&stg_r[0], (void**)&stg_r[1], (void**)&visits,
+        (void**)&owners, (void**)&own_viol};
     for (void* ptr : fresh) {
       for (void** m : members)
         if (*m == ptr) *m = nullptr;
@@ -878,6 +898,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->lr_rule < 0 || p->lr_rule > 1 || !(p->ada_eps >= 0.f)) return MF_E_INVAL;
   if (p->exact_order < 0 || p->exact_order > 1) return MF_E_INVAL;
   if (p->group_cols < 0 || p->group_cols > 1) return MF_E_INVAL;
+  if (p->check_owners < 0 || p->check_owners > 1) return MF_E_INVAL;
   if (p->group_cols && (p->schedule != MF_HOGWILD || p->rating_stage || p->prefetch > 1))
     return MF_E_UNSUPPORTED;
   if (p->rating_stage < 0 || p->rating_stage > 1) return MF_E_INVAL;
@@ -1098,6 +1119,12 @@ static mf_status alloc_schedule(mf_ctx* c) {
     TRY(c->alloc(&c->seq, (size_t)cap));
     TRY(c->alloc(&c->rank_arr, (size_t)cap));
     TRY(c->alloc(&c->tickets, (size_t)c->c));
+    if (c->p.check_owners) {
+      TRY(c->alloc(&c->owners, (size_t)c->c));
+      TRY(c->alloc(&c->own_viol, 1));
+      CUDA_TRY(c, cudaMemsetAsync(c->owners, 0xFF, (size_t)c->c * 4, c->st));   // all free (-1)
+      CUDA_TRY(c, cudaMemsetAsync(c->own_viol, 0, 4, c->st));
+    }
     if (c->p.cyclic) {
       TRY(c->alloc(&c->tau, (size_t)(nb * c->c)));
       TRY(c->alloc(&c->sigma, (size_t)(nb * c->c)));
@@ -1263,7 +1290,10 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
   int32_t *ou, *ov;
   float* orr;
   TRY(stage_input(c, N, u, v, r, on_device, &du, &dv, &dr, &ou, &ov, &orr));
-  TRY(validate(c, N, du, dv, dr));
+  {
+    Nvtx rv("validate");
+    TRY(validate(c, N, du, dv, dr));
+  }
 
   // relabel (A: S_ROW, S_COL) first: a rank only needs the ratings of the row segments it owns
   TRY(relabel(c, kTagRow, c->m, &c->rho_r));
@@ -1295,6 +1325,7 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
   // Alg. 1 l.2 random_shuffle: storage order = perm(S_SHUF, N) over caller indices.
   // A rank sorts only its own ratings by the same keys: their relative order is the global one.
   {
+    Nvtx rs("shuffle (Alg. 1 l.2)");
     uint64_t *k0 = nullptr, *k1 = nullptr;
     uint32_t* v0 = nullptr;
     TRY(c->alloc(&k0, (size_t)N));
@@ -1445,7 +1476,10 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
       KERNEL_TRY(c);
     }
   }
-  TRY(init_factors(c));
+  {
+    Nvtx ri("init P, Q (Alg. 1 l.3)");
+    TRY(init_factors(c));
+  }
   if (c->p.lr_rule == 1) {
     TRY(c->alloc(&c->GP, (size_t)(c->m * c->k)));
     TRY(c->alloc(&c->GQ, (size_t)(c->n * c->k)));
@@ -1494,6 +1528,7 @@ static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, cons
   std::vector<std::vector<Rating>> hr((size_t)nb);
   std::vector<int64_t> bcount((size_t)nb, 0);
   {  // ---- pass 1
+    Nvtx rp1("out-of-core pass 1 (chunks of %lld)", (long long)C);
     int32_t *cu = nullptr, *cv = nullptr;
     float* cr = nullptr;
     uint32_t *b0 = nullptr, *b1 = nullptr, *i0 = nullptr, *i1 = nullptr;
@@ -1593,6 +1628,7 @@ static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, cons
   if (want_dup) CUDA_TRY(c, cudaMallocHost(&c->h_dup, ns * sizeof(uint16_t)));
   // ---- pass 2
   {
+    Nvtx rp2("out-of-core pass 2 (per block)");
     Grid Gd{c->m, c->n, c->a, c->s, c->c, c->wf};
     const int64_t per = (int64_t)c->s * c->c;
     uint64_t *k0 = nullptr, *k1 = nullptr;
@@ -1769,6 +1805,7 @@ mf_status mf_load_coo(mf_ctx* c, int32_t set, int64_t nnz, const int32_t* u, con
   TRY(c->enter());
   if (nnz < 0 || (nnz > 0 && (!u || !v || !r))) return c->fail(MF_E_INVAL, "bad COO arguments");
   const std::vector<std::pair<void*, size_t>> before = c->sizes;
+  Nvtx range("mf_load_coo(%s, N=%lld)", set == MF_TRAIN ? "train" : "test", (long long)nnz);
   mf_status s = MF_OK;
   if (set == MF_TRAIN) {
     if (c->train_loaded) return c->fail(MF_E_STATE, "train set already loaded");
@@ -1999,6 +2036,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     if (L.ada.GP) L.g = c->p.alpha;
     L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
     L.visits = c->visits + base; L.upd = c->upd_dev;
+    L.owners = c->owners; L.viol = c->own_viol;
     // Diagnostics only (MF_PROFILE_WAVES=1): per-worker clock64 totals of ticket waits and
     // sub-block runs, summarised on stderr after the launch (synchronises).
     static const bool kProfWaves = std::getenv("MF_PROFILE_WAVES") != nullptr;
@@ -2127,6 +2165,7 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   TRY(c->enter());
   if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
   const int32_t t = c->t;
+  Nvtx range("epoch %d", t);
   const float g = gamma_of(c->p.alpha, c->p.beta, t);   // Eq. 9
   c->n_sgd = 0;
   c->n_launch = 0;
@@ -2136,14 +2175,17 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   CUDA_TRY(c, cudaEventRecord(c->ev_e0, c->st));
   CUDA_TRY(c, cudaEventRecord(c->ev_s0, c->st));
   const bool hog = !c->wf && !c->libmf && c->ch_off.back() > 0;
-  if (hog && c->prebuilt_t == t) {          // built on the side stream during the last epoch
-    TRY(join_side(c));
-    std::swap(c->chunk_order, c->chunk_order_alt);
-    c->sched_built_for = t;
-  } else {
-    TRY(build_schedule(c, t));
+  {
+    Nvtx rsched("schedule build");
+    if (hog && c->prebuilt_t == t) {        // built on the side stream during the last epoch
+      TRY(join_side(c));
+      std::swap(c->chunk_order, c->chunk_order_alt);
+      c->sched_built_for = t;
+    } else {
+      TRY(build_schedule(c, t));
+    }
+    c->prebuilt_t = -1;
   }
-  c->prebuilt_t = -1;
   if (hog) {
     if (!c->ev_ss_go) CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_ss_go, cudaEventDisableTiming));
     CUDA_TRY(c, cudaEventRecord(c->ev_ss_go, c->st));
@@ -2196,11 +2238,15 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   CUDA_TRY(c, cudaEventRecord(c->ev_c0, c->st));
   CUDA_TRY(c, cudaEventRecord(c->ev_c1, c->st));
   for (int j = 0; j < c->a; ++j) {
+    Nvtx rj("sub-epoch %d", j);
     int32_t nb = 0, nx = 0;
     if (mf_strata_plan(c->p.seed, c->a, c->G, c->rank, c->n, t, j, hold, blocks.data(), &nb,
                        xf.data(), &nx) != MF_OK)
       return c->fail(MF_E_INVAL, "strata plan failed");
-    TRY(rotate_q(c, xf.data(), nx));
+    if (nx) {
+      Nvtx rq("Q rotation (%d segments)", nx);
+      TRY(rotate_q(c, xf.data(), nx));
+    }
     if (c->G > 1) c->comm->set_holders(hold, c->a);
     int buf = 0;
     if (c->staged) {
@@ -2340,6 +2386,7 @@ mf_status mf_rmse(mf_ctx* c, int32_t set, double* out) {
   }
   if (set == MF_TRAIN && (c->G > 1 || c->staged))
     return c->fail(MF_E_UNSUPPORTED, "train-set RMSE needs resident single-GPU ratings");
+  Nvtx range("mf_rmse(%s)", set == MF_TRAIN ? "train" : "test");
   // world > 1: every rank evaluates the test samples of the row segments it owns (filtered at
   // load) against a complete Q, then the SSE and count are summed over ranks.
   if (c->G > 1) TRY(gather_q(c));
@@ -2361,6 +2408,42 @@ mf_status mf_rmse(mf_ctx* c, int32_t set, double* out) {
   const double rmse = (double)c->p.rating_scale * std::sqrt(sse / std::max(cnt, 1.0));
   *out = cnt > 0 ? rmse : 0.0;     // global count when world > 1 (all-reduced above)
   if (std::isnan(*out)) return c->fail(MF_E_RANGE, "RMSE is NaN (divergence)");
+  return MF_OK;
+}
+
+mf_status mf_owner_violations(mf_ctx* c, int64_t* out) {
+  if (!c || !out) return MF_E_INVAL;
+  TRY(c->enter());
+  if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
+  if (!c->own_viol) return c->fail(MF_E_STATE, "create the ctx with check_owners = 1 (wavefront)");
+  unsigned h = 0;
+  CUDA_TRY(c, cudaMemcpyAsync(&h, c->own_viol, 4, cudaMemcpyDeviceToHost, c->st));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  *out = h;
+  return MF_OK;
+}
+
+mf_status mf_loss(mf_ctx* c, double* out) {
+  if (!c || !out) return MF_E_INVAL;
+  TRY(c->enter());
+  if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
+  if (c->staged) return c->fail(MF_E_UNSUPPORTED, "the loss needs resident ratings");
+  Nvtx range("mf_loss");
+  if (c->G > 1) TRY(gather_q(c));
+  RmseLaunch L{};
+  L.storage = c->p.storage; L.k = c->k; L.test = c->slots; L.N = c->nslots; L.P = c->P; L.Q = c->Q;
+  L.partial = c->rm_partial; L.out = c->rm_out; L.num_sms = c->num_sms; L.stream = c->st;
+  L.loss = 1; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q;
+  CUDA_TRY(c, launch_rmse(L));
+  if (c->G > 1) {                        // every rank holds the ratings of its own row segments
+    std::string why;
+    if (!c->comm->allreduce_sum(c->rm_out, 1, &why)) return c->fail(MF_E_NCCL, "loss: %s", why.c_str());
+  }
+  double h = 0.0;
+  CUDA_TRY(c, cudaMemcpyAsync(&h, c->rm_out, 8, cudaMemcpyDeviceToHost, c->st));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  *out = h;
+  if (std::isnan(h)) return c->fail(MF_E_RANGE, "loss is NaN (divergence)");
   return MF_OK;
 }
 

@@ -69,6 +69,8 @@ struct WavefrontLaunch {
                             // fence} clock64 totals, or nullptr
   unsigned* visits;         // s*c per strata block: visits of sub-block (i, j) (one atomic per wave)
   unsigned long long* upd;  // samples updated (device count)
+  int* owners;              // params.check_owners: c column tags (-1 = free), else nullptr
+  unsigned* viol;           // mutual-exclusion violations found by the checker
   cudaStream_t stream;
   int *out_lanes, *out_grid;
 };
@@ -80,6 +82,8 @@ struct RmseLaunch {
   const void *P, *Q;
   double* partial;  // num_sms*4
   double* out;      // 1
+  int loss;         // 1: Eq. 2 (squared error + lp ||p||^2 + lq ||q||^2) instead of squared error
+  float lp, lq;
   int num_sms;
   cudaStream_t stream;
 };

@@ -139,6 +139,18 @@ __device__ __forceinline__ void ticket_release(int* t, int next, unsigned gmask,
   if (gl == 0) st_relaxed(t, next);
 }
 
+// Debug ownership checker (params.check_owners; SURVEY 5 race detection): a worker tags the
+// column block it acquires (atomicCAS from -1) and clears the tag on release (atomicExch back);
+// any tag it finds set by another worker, or not its own on release, is a mutual-exclusion
+// violation of the ticket protocol on the global P/Q rows (which compute-sanitizer's racecheck,
+// shared memory only, cannot see).  Row blocks are private to their worker by construction.
+__device__ __forceinline__ void own_acquire(int* owners, unsigned* viol, int col, int worker) {
+  if (owners && atomicCAS(owners + col, -1, worker) != -1) atomicAdd(viol, 1u);
+}
+__device__ __forceinline__ void own_release(int* owners, unsigned* viol, int col, int worker) {
+  if (owners && atomicExch(owners + col, -1) != worker) atomicAdd(viol, 1u);
+}
+
 template <typename T, int K, int L, bool ADA, bool EX>
 __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ slots,
                                                    const int64_t* __restrict__ sub_off,
@@ -148,7 +160,9 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
                                                    T* __restrict__ P, T* __restrict__ Q, Step st,
                                                    int64_t shift, AdaArgs ada,
                                                    unsigned* __restrict__ visits,
-                                                   unsigned long long* __restrict__ upd) {
+                                                   unsigned long long* __restrict__ upd,
+                                                   int* __restrict__ owners,
+                                                   unsigned* __restrict__ viol) {
   const int lane = threadIdx.x & 31;
   const int grp = lane / L, gl = lane % L, gbase = grp * L;
   const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
@@ -161,11 +175,13 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
     const int col = __ldg(my_seq + w);
     const int tgt = __ldg(my_rank + w);
     ticket_acquire(tickets + col, tgt);
+    if (gl == 0) own_acquire(owners, viol, col, worker);
     const int64_t sb = (int64_t)worker * c + col;
     const int64_t lo = __ldg(sub_off + sb) + shift;
     done += run_serial<T, K, L, 2, false, ADA, EX>(slots, lo, (int)(__ldg(sub_off + sb + 1) + shift - lo),
                                                true, P, Q, st, gl, gbase, gmask, ada);
     if (gl == 0) atomicAdd(visits + sb, 1u);
+    if (gl == 0) own_release(owners, viol, col, worker);
     ticket_release(tickets + col, tgt + 1, gmask, gl);
   }
   if (gl == 0 && done) atomicAdd(upd, (unsigned long long)done);
@@ -185,7 +201,9 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
                                                     int64_t shift,
                                                     long long* __restrict__ prof,
                                                     unsigned* __restrict__ visits,
-                                                    unsigned long long* __restrict__ upd) {
+                                                    unsigned long long* __restrict__ upd,
+                                                    int* __restrict__ owners,
+                                                    unsigned* __restrict__ viol) {
   extern __shared__ __align__(16) char smem[];
   constexpr int ROWB = K * (int)sizeof(T);
   const int lane = threadIdx.x & 31;
@@ -231,6 +249,7 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     const long long tw0 = prof ? clock64() : 0;
     if (!ready) {
       ticket_acquire(tickets + col0, tgt0);   // relaxed spin + fence.acq_rel
+      if (gl == 0) own_acquire(owners, viol, col0, worker);
       if (n0 > 0)
         run_subblock_ring<T, K, L, RS, F, EX>(slots, dup, lo0, n0, h0, P, Q, st, gl, gbase,
                                           gmask, ring, true, false);
@@ -255,12 +274,14 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     // next column already released: issue its row prefetch BEFORE this wave's release fence.
     // (Its p rows may have been stored by this sub-block: same thread, issued after them.)
     ready = w + 1 < c && poll1 == tgt1;
+    if (ready && gl == 0) own_acquire(owners, viol, col1, worker);
     if (ready && n1 > 0)
       run_subblock_ring<T, K, L, RS, F, EX>(slots, dup, lo1, n1, h1, P, Q, st, gl, gbase, gmask,
                                         ring, true, false);
     const long long tw2 = prof ? clock64() : 0;
     if (gl == 0) atomicAdd(visits + (int64_t)worker * c + col0, 1u);   // sub-block (worker, col0)
     n_upd += n0;
+    if (gl == 0) own_release(owners, viol, col0, worker);
     ticket_release(tickets + col0, tgt0 + 1, gmask, gl);   // fence; syncwarp; relaxed store
     if (prof) {
       t_wait += tw1 - tw0;
@@ -366,10 +387,12 @@ __global__ void __launch_bounds__(32) k_libmf(const Rating* __restrict__ slots,
 // reduction to one partial per CTA; k_rmse_final sums the partials in a fixed order.
 // ---------------------------------------------------------------------------------------------
 template <typename T, int K, int L>
+// loss = 1: Eq. 2 instead: per sample (r - p.q)^2 + lp ||p_u||^2 + lq ||q_v||^2.
 __global__ void __launch_bounds__(256) k_rmse_partial(const Rating* __restrict__ test, int64_t N,
                                                       const T* __restrict__ P,
                                                       const T* __restrict__ Q,
-                                                      double* __restrict__ partial) {
+                                                      double* __restrict__ partial, int loss,
+                                                      float lp, float lq) {
   using G = Geo<T, K, L>;
   constexpr int PW = Pack<T>::kPerWord;
   const int lane = threadIdx.x & 31;
@@ -392,13 +415,26 @@ __global__ void __launch_bounds__(256) k_rmse_partial(const Rating* __restrict__
       Pack<T>::unpack(pw.w[i], p + i * PW);
       Pack<T>::unpack(qw.w[i], q + i * PW);
     }
-    float d = 0.f;
+    float d = 0.f, pp = 0.f, qq = 0.f;
 #pragma unroll
-    for (int e = 0; e < G::VEC; ++e) d = fmaf(p[e], q[e], d);
+    for (int e = 0; e < G::VEC; ++e) {
+      d = fmaf(p[e], q[e], d);
+      pp = fmaf(p[e], p[e], pp);
+      qq = fmaf(q[e], q[e], qq);
+    }
 #pragma unroll
-    for (int o = L / 2; o > 0; o >>= 1) d += __shfl_xor_sync(gmask, d, o);
+    for (int o = L / 2; o > 0; o >>= 1) {
+      d += __shfl_xor_sync(gmask, d, o);
+      if (loss) {
+        pp += __shfl_xor_sync(gmask, pp, o);
+        qq += __shfl_xor_sync(gmask, qq, o);
+      }
+    }
     const float e = r - d;
-    if (gl == 0) acc += (double)e * (double)e;
+    if (gl == 0) {
+      acc += (double)e * (double)e;
+      if (loss) acc += (double)lp * (double)pp + (double)lq * (double)qq;
+    }
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
@@ -516,8 +552,10 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
   AdaArgs ada = a.ada;
   unsigned* visits = a.visits;
   unsigned long long* upd = a.upd;
+  int* owners = a.owners;
+  unsigned* viol = a.viol;
   void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &st, &shift,
-                  &ada, &visits, &upd};
+                  &ada, &visits, &upd, &owners, &viol};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, 0,
                                      a.stream);
 }
@@ -556,8 +594,10 @@ static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
   long long* prof = a.prof;
   unsigned* visits = a.visits;
   unsigned long long* upd = a.upd;
+  int* owners = a.owners;
+  unsigned* viol = a.viol;
   void* args[] = {&slots, &dup, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &st,
-                  &shift, &prof, &visits, &upd};
+                  &shift, &prof, &visits, &upd, &owners, &viol};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, smem,
                                      a.stream);
 }
@@ -578,7 +618,8 @@ static cudaError_t launch_rmse_t(const RmseLaunch& a) {
   const int blocks = a.num_sms * 4;
   if (a.N > 0)
     k_rmse_partial<T, K, L><<<blocks, threads, 0, a.stream>>>(
-        a.test, a.N, reinterpret_cast<const T*>(a.P), reinterpret_cast<const T*>(a.Q), a.partial);
+        a.test, a.N, reinterpret_cast<const T*>(a.P), reinterpret_cast<const T*>(a.Q), a.partial,
+        a.loss, a.lp, a.lq);
   else
     cudaMemsetAsync(a.partial, 0, sizeof(double) * blocks, a.stream);
   k_rmse_final<<<1, 256, 0, a.stream>>>(a.partial, blocks, a.out);

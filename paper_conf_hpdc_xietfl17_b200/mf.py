@@ -56,7 +56,7 @@ class Params(ctypes.Structure):
                 ("stream", ctypes.c_void_p), ("alloc", ctypes.POINTER(Allocator)),
                 ("launch_blocks", ctypes.c_int32), ("exact_order", ctypes.c_int32),
                 ("rating_stage", ctypes.c_int32), ("stage_chunk", ctypes.c_int64),
-                ("group_cols", ctypes.c_int32)]
+                ("group_cols", ctypes.c_int32), ("check_owners", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -70,8 +70,9 @@ class Stats(ctypes.Structure):
 
 _lib = None
 EXPORTED = ["mf_abi_version", "mf_params_default", "mf_create", "mf_load_coo", "mf_train_epoch",
-            "mf_rmse", "mf_get_factors", "mf_set_factors", "mf_set_epoch", "mf_get_epoch",
+            "mf_rmse", "mf_loss", "mf_get_factors", "mf_set_factors", "mf_set_epoch", "mf_get_epoch",
             "mf_export_schedule", "mf_get_stats", "mf_get_launch_ms", "mf_check_visits",
+            "mf_owner_violations",
             "mf_strata_holders", "mf_strata_plan",
             "mf_destroy",
             "mf_last_error", "mf_status_string"]
@@ -94,6 +95,7 @@ def lib() -> ctypes.CDLL:
         "mf_load_coo": (i32, [vp, i32, i64, vp, vp, vp, i32]),
         "mf_train_epoch": (i32, [vp, ctypes.POINTER(i32)]),
         "mf_rmse": (i32, [vp, i32, ctypes.POINTER(ctypes.c_double)]),
+        "mf_loss": (i32, [vp, ctypes.POINTER(ctypes.c_double)]),
         "mf_get_factors": (i32, [vp, vp, vp, i32]),
         "mf_set_factors": (i32, [vp, vp, vp, i32]),
         "mf_set_epoch": (i32, [vp, i32]),
@@ -102,6 +104,7 @@ def lib() -> ctypes.CDLL:
         "mf_get_stats": (i32, [vp, ctypes.POINTER(Stats)]),
         "mf_get_launch_ms": (i32, [vp, vp, ctypes.POINTER(i64)]),
         "mf_check_visits": (i32, [vp, ctypes.POINTER(i64), ctypes.POINTER(i64), ctypes.POINTER(i32)]),
+        "mf_owner_violations": (i32, [vp, ctypes.POINTER(i64)]),
         "mf_strata_holders": (i32, [u64, i32, i32, i32, i32, vp]),
         "mf_strata_plan": (i32, [u64, i32, i32, i32, i64, i32, i32, vp, vp, vp, vp, vp]),
         "mf_destroy": (None, [vp]),
@@ -202,7 +205,7 @@ class MF:
                  lane_bytes: int = 0, prefetch: int = 0, wf_kernel: int = 0, staged: bool = False,
                  lr_rule: str = "eq9", ada_eps: float = 1e-8, launch_blocks: int = 0,
                  exact_order: bool = False, rating_stage: int = 0, stage_chunk: int = 0,
-                 group_cols: bool = False,
+                 group_cols: bool = False, check_owners: bool = False,
                  device: int = 0, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, transport: int = 0, stream=None,
                  allocator: str = "torch", device_budget: int | None = None):
@@ -223,6 +226,7 @@ class MF:
         p.rating_stage = int(rating_stage)
         p.stage_chunk = int(stage_chunk)
         p.group_cols = int(group_cols)
+        p.check_owners = int(check_owners)
         p.lr_rule, p.ada_eps = {"eq9": 0, "adagrad": 1}[lr_rule], ada_eps
         p.device, p.rank, p.world, p.transport = device, rank, world, transport
         self._id_buf = None
@@ -291,6 +295,12 @@ class MF:
         self._check(lib().mf_rmse(self.h, SETS[set], ctypes.byref(out)), "mf_rmse")
         return out.value
 
+    def loss(self) -> float:
+        """Eq. 2 over the training set (scaled rating units)."""
+        out = ctypes.c_double(0)
+        self._check(lib().mf_loss(self.h, ctypes.byref(out)), "mf_loss")
+        return out.value
+
     def factors(self, on_device: bool = False):
         if on_device:
             torch = _torch()
@@ -350,6 +360,12 @@ class MF:
         """High-water mark of the ctx's device memory (torch allocator hooks only)."""
         return self._alloc.peak if self._alloc is not None else -1
 
+    def owner_violations(self) -> int:
+        """Ownership-checker violations since load (check_owners = True, wavefront)."""
+        n = ctypes.c_int64(0)
+        self._check(lib().mf_owner_violations(self.h, ctypes.byref(n)), "mf_owner_violations")
+        return n.value
+
     def stats(self) -> dict:
         s = Stats()
         self._check(lib().mf_get_stats(self.h, ctypes.byref(s)), "mf_get_stats")
@@ -390,6 +406,10 @@ def mf_rmse(ctx: MF, set: str = "test") -> float:
     return ctx.rmse(set)
 
 
+def mf_loss(ctx: MF) -> float:
+    return ctx.loss()
+
+
 def mf_get_factors(ctx: MF, on_device: bool = False):
     return ctx.factors(on_device)
 
@@ -420,6 +440,10 @@ def mf_get_launch_ms(ctx: MF) -> np.ndarray:
 
 def mf_check_visits(ctx: MF) -> dict:
     return ctx.check_visits()
+
+
+def mf_owner_violations(ctx: MF) -> int:
+    return ctx.owner_violations()
 
 
 def mf_last_error(ctx: MF) -> str:

@@ -483,6 +483,61 @@ def test_rmse_kernel_against_numpy(tiny):
     assert abs(g.rmse("train") - wantt) <= 1e-5 * wantt
 
 
+@pytest.mark.parametrize("kw", [dict(schedule="hogwild", workers=1), dict(schedule="hogwild", grid_a=4),
+                                dict(schedule="wavefront", workers=8, wf_cols=16, storage="fp16")])
+def test_loss_kernel_against_the_oracle(tiny, kw):
+    """mf_loss = Eq. 2 over the training set (oracle or_loss: double dots and norms) on the same
+    factors: the oracle's, copied in (so only the reduction differs)."""
+    g, o = pair(tiny, **TABLE3_NETFLIX, **kw)
+    o.train_epoch()
+    Po, Qo = o.factors()
+    g.set_factors(Po, Qo)
+    lg, lo = g.loss(), o.loss()
+    assert abs(lg - lo) <= 1e-5 * lo, (lg, lo)
+
+
+def test_per_epoch_metrics_lines(tiny):
+    """SURVEY 5 metrics: one JSON line per epoch with updates/s, algorithmic GB/s, % of the HBM
+    roofline, test RMSE and the Eq. 2 loss, all from the library; the loss decreases."""
+    import io
+    import json
+    from paper_conf_hpdc_xietfl17_b200 import metrics
+    g = mf.MF(tiny.m, tiny.n, 16, storage="fp16", **TABLE3_NETFLIX)
+    g.load(tiny.u, tiny.v, tiny.r)
+    g.load(tiny.ut, tiny.vt, tiny.rt, "test")
+    buf = io.StringIO()
+    lines = metrics.train(g, 3, out=buf)
+    parsed = [json.loads(x) for x in buf.getvalue().splitlines()]
+    assert parsed == json.loads(json.dumps(lines))
+    assert [x["epoch"] for x in parsed] == [0, 1, 2]
+    for x in parsed:
+        assert x["updates"] == tiny.N and x["updates_per_s"] > 0 and x["pct_hbm_roofline"] > 0
+        assert x["alg_GBps"] == pytest.approx(x["updates_per_s"] * (12 + 4 * 16 * 2) / 1e9)
+    assert parsed[2]["train_loss"] < parsed[0]["train_loss"]
+    assert parsed[2]["test_rmse"] < parsed[0]["test_rmse"]
+
+
+@pytest.mark.parametrize("kw", [dict(workers=8, wf_cols=16), dict(workers=8, wf_cols=16, cyclic=True),
+                                dict(workers=8, wf_cols=16, wf_kernel=2),
+                                dict(workers=5, wf_cols=7, grid_a=4, k=128, storage="fp16")])
+def test_ownership_checker_finds_no_overlap(tiny, kw):
+    """SURVEY 5 race detection for the deterministic mode: with check_owners every wave tags
+    its column block on acquire and clears it on release; across 3 epochs no two workers ever
+    held a column block at once, and the checked run equals the unchecked one bit for bit."""
+    kw = dict(kw)
+    k = kw.pop("k", 16)
+    out = []
+    for chk in (True, False):
+        g = mf.MF(tiny.m, tiny.n, k, schedule="wavefront", check_owners=chk, **kw)
+        g.load(tiny.u, tiny.v, tiny.r)
+        for _ in range(3):
+            g.train_epoch()
+        if chk:
+            assert g.owner_violations() == 0
+        out.append(g.factors())
+    assert np.array_equal(out[0][0], out[1][0]) and np.array_equal(out[0][1], out[1][1])
+
+
 def test_set_factors_rounds_like_the_oracle(tiny):
     rng = np.random.default_rng(4)
     P = rng.normal(size=(tiny.m, 16)).astype(np.float32)
