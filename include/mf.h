@@ -100,7 +100,13 @@ typedef struct mf_params {
                              G += g^2, step alpha*g/sqrt(G + ada_eps); Hogwild and register
                              wavefront kernels                                                  */
   float ada_eps;          /* ADAGRAD epsilon (0 = 1e-8)                                         */
-  int32_t staged;         /* 1 = out-of-core ratings (section 6.2): the bucketed
+  int32_t staged;         /* 2 = ratings AND P out of core (section 6.1 step 3, and the
+                             three streams of section 6.3): P's row segments live in
+                             pinned host memory and the strata blocks run one at a time, each
+                             with its segment copied in on a copy stream, trained, and written
+                             back on a D2H stream while the next block computes; Q stays
+                             resident.  One GPU, Eq. 9 step; same result as resident.
+                             1 = out-of-core ratings (section 6.2): the bucketed
                              ratings live in pinned host memory (a host train set is
                              preprocessed in chunks of stage_chunk samples, never whole in
                              HBM; a device set is preprocessed resident, then moved) and

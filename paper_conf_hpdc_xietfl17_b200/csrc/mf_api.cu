@@ -272,6 +272,27 @@ template <> __device__ __forceinline__ __nv_bfloat16 from_f32<__nv_bfloat16>(flo
   return __float2bfloat16_rn(x);
 }
 
+// inv[rho[i]] = i (relabelled row -> original id)
+__global__ void k_invert(const int32_t* __restrict__ rho, int64_t n, int32_t* __restrict__ inv) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    inv[rho[i]] = (int32_t)i;
+}
+
+// Alg. 1 l.3 for relabelled rows [lo, lo + rows) into a segment buffer (staged == 2): the same
+// value as k_init for every (id, d), id = inv[row].
+template <typename T>
+__global__ void k_init_rows(T* __restrict__ X, const int32_t* __restrict__ inv, int64_t lo,
+                            int64_t rows, int k, uint64_t S, float amp) {
+  const int64_t total = rows * k;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t id = inv[lo + x / k], d = x % k;
+    const float u01 = (float)(hkey(S, (uint64_t)(id * k + d)) >> 40) * 0x1p-24f;
+    X[x] = static_cast<T>(u01 * amp);
+  }
+}
+
 // model_shuffle (Alg. 1 l.15): out[id][d] = fp32(X[rho[id]][d])
 template <typename T>
 __global__ void k_unrelabel(const T* __restrict__ X, const int32_t* __restrict__ rho, int64_t rows,
@@ -512,6 +533,15 @@ __global__ void k_permute_slots(const uint32_t* __restrict__ order, int64_t n,
   }
 }
 
+__global__ void k_test_seg(const Rating* __restrict__ t, int64_t N, int64_t m, int64_t a,
+                           uint32_t* __restrict__ seg, uint32_t* __restrict__ idx) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < N;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    seg[i] = (uint32_t)((int64_t)t[i].u * a / m);
+    idx[i] = (uint32_t)i;
+  }
+}
+
 __global__ void k_iota_u32(uint32_t* __restrict__ x, int64_t n) {
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < n;
        j += (int64_t)gridDim.x * blockDim.x)
@@ -659,6 +689,18 @@ struct mf_ctx {
   int64_t staged_t = -1, staged_j = -1;
   int cur_buf = 0;
   int64_t h2d_bytes = 0;
+  // staged == 2 (section 6.1 step 3): P is out of core too.  Its row segments live
+  // in pinned host memory and one strata block at a time is trained with its segment staged
+  // into one of two device slots: copy-in stream cs, compute stream st, write-back stream ds
+  // (the three streams of section 6.3).  Q stays resident.
+  bool pq = false;
+  char* h_P = nullptr;
+  char* Pslot[2] = {nullptr, nullptr};
+  int64_t pseg_max = 0;
+  cudaStream_t ds = nullptr;
+  cudaEvent_t ev_pin[2] = {nullptr, nullptr}, ev_pcomp[2] = {nullptr, nullptr};
+  cudaEvent_t ev_pout[2] = {nullptr, nullptr};
+  std::vector<int64_t> test_seg_off;   // pq: test ratings grouped by row segment (a + 1)
 
   mf_status fail(mf_status s, const char* fmt, ...) {
     char buf[512];
@@ -759,7 +801,7 @@ struct mf_ctx {
         (void**)&lm_rem, (void**)&stg[0], (void**)&stg[1], (void**)&stg_dup[0],
         (void**)&stg_dup[1], (void**)&stg_u[0], (void**)&stg_u[1], (void**)&stg_v16[0],
         (void**)&stg_v16[1], (void**)&stg_r[0], (void**)&stg_r[1], (void**)&visits,
-        (void**)&owners, (void**)&own_viol};
+        (void**)&owners, (void**)&own_viol, (void**)&Pslot[0], (void**)&Pslot[1]};
     for (void* ptr : fresh) {
       for (void** m : members)
         if (*m == ptr) *m = nullptr;
@@ -768,7 +810,8 @@ struct mf_ctx {
       if (ptr == tmp) tmp = nullptr;
     }
     if (!tmp) tmp_bytes = 0;
-    for (void** h : {(void**)&h_slots, (void**)&h_u, (void**)&h_v16, (void**)&h_r, (void**)&h_dup})
+    for (void** h : {(void**)&h_slots, (void**)&h_u, (void**)&h_v16, (void**)&h_r, (void**)&h_dup,
+                     (void**)&h_P})
       if (*h) { cudaFreeHost(*h); *h = nullptr; }
     cudaGetLastError();
   }
@@ -894,7 +937,9 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->prefetch < 0 || p->prefetch > 2) return MF_E_INVAL;
   if (p->wf_kernel < 0 || p->wf_kernel > 2 || p->launch_blocks < 0) return MF_E_INVAL;
   if (p->transport < 0 || p->transport > 1) return MF_E_INVAL;
-  if (p->staged < 0 || p->staged > 1) return MF_E_INVAL;
+  if (p->staged < 0 || p->staged > 2) return MF_E_INVAL;
+  if (p->staged == 2 && (p->world > 1 || p->lr_rule != 0 || p->schedule == MF_LIBMF))
+    return MF_E_UNSUPPORTED;                     // P out of core: one GPU, Eq. 9 step
   if (p->lr_rule < 0 || p->lr_rule > 1 || !(p->ada_eps >= 0.f)) return MF_E_INVAL;
   if (p->exact_order < 0 || p->exact_order > 1) return MF_E_INVAL;
   if (p->group_cols < 0 || p->group_cols > 1) return MF_E_INVAL;
@@ -927,7 +972,8 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   c->f = p->batch_f > 0 ? p->batch_f : 256;
   c->wf = p->schedule == MF_WAVEFRONT;
   c->libmf = p->schedule == MF_LIBMF;
-  c->staged = p->staged == 1;
+  c->staged = p->staged >= 1;
+  c->pq = p->staged == 2;
   if (c->wf) {
     const int64_t rows_per_seg = p->m / a;
     int64_t s = p->workers > 0 ? p->workers : std::min<int64_t>(768, std::max<int64_t>(1, rows_per_seg / 4));
@@ -993,6 +1039,7 @@ void mf_destroy(mf_ctx* c) {
   // stratum's H2D into a staging buffer on cs, which nothing on st waits for) and st itself
   if (c->ss) cudaStreamSynchronize(c->ss);
   if (c->cs) cudaStreamSynchronize(c->cs);
+  if (c->ds) cudaStreamSynchronize(c->ds);
   if (c->st) cudaStreamSynchronize(c->st);
   std::vector<std::pair<void*, size_t>> all = c->sizes;
   for (auto& x : all) {
@@ -1009,6 +1056,11 @@ void mf_destroy(mf_ctx* c) {
   if (c->h_v16) cudaFreeHost(c->h_v16);
   if (c->h_r) cudaFreeHost(c->h_r);
   if (c->h_dup) cudaFreeHost(c->h_dup);
+  if (c->h_P) cudaFreeHost(c->h_P);
+  for (int i = 0; i < 2; ++i)
+    for (cudaEvent_t e : {c->ev_pin[i], c->ev_pcomp[i], c->ev_pout[i]})
+      if (e) cudaEventDestroy(e);
+  if (c->ds) cudaStreamDestroy(c->ds);
   for (int i = 0; i < 2; ++i) {
     if (c->ev_h2d[i]) cudaEventDestroy(c->ev_h2d[i]);
     if (c->ev_free[i]) cudaEventDestroy(c->ev_free[i]);
@@ -1084,12 +1136,59 @@ static void launch_init(mf_ctx* c, void* X, const int32_t* rho, int64_t rows, ui
   k_init<T><<<grid_for(rows * c->k, c->num_sms), 256, 0, c->st>>>((T*)X, rho, rows, c->k, S, amp);
 }
 
+template <typename T>
+static void launch_init_rows(mf_ctx* c, void* X, const int32_t* inv, int64_t lo, int64_t rows,
+                             uint64_t S, float amp) {
+  k_init_rows<T><<<grid_for(rows * c->k, c->num_sms), 256, 0, c->st>>>((T*)X, inv, lo, rows, c->k,
+                                                                         S, amp);
+}
+
+// staged == 2: P initialised segment by segment in a device slot and written to pinned host
+// memory; the two device slots of one row segment each are all the HBM P ever takes.
+static mf_status init_p_out_of_core(mf_ctx* c, float amp, uint64_t SP) {
+  const size_t rowb = (size_t)c->k * c->ssize();
+  c->pseg_max = 0;
+  for (int r = 0; r < c->a; ++r)
+    c->pseg_max = std::max(c->pseg_max, cdiv64((int64_t)(r + 1) * c->m, c->a) - cdiv64((int64_t)r * c->m, c->a));
+  CUDA_TRY(c, cudaMallocHost(&c->h_P, (size_t)c->m * rowb));
+  TRY(c->alloc(&c->Pslot[0], (size_t)c->pseg_max * rowb));
+  TRY(c->alloc(&c->Pslot[1], (size_t)c->pseg_max * rowb));
+  int32_t* inv = nullptr;
+  TRY(c->alloc(&inv, (size_t)c->m));
+  k_invert<<<grid_for(c->m, c->num_sms), 256, 0, c->st>>>(c->rho_r, c->m, inv);
+  KERNEL_TRY(c);
+  for (int r = 0; r < c->a; ++r) {
+    const int64_t lo = cdiv64((int64_t)r * c->m, c->a), hi = cdiv64((int64_t)(r + 1) * c->m, c->a);
+    switch (c->p.storage) {
+      case MF_FP32: launch_init_rows<float>(c, c->Pslot[0], inv, lo, hi - lo, SP, amp); break;
+      case MF_FP16: launch_init_rows<__half>(c, c->Pslot[0], inv, lo, hi - lo, SP, amp); break;
+      default: launch_init_rows<__nv_bfloat16>(c, c->Pslot[0], inv, lo, hi - lo, SP, amp); break;
+    }
+    KERNEL_TRY(c);
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_P + (size_t)lo * rowb, c->Pslot[0], (size_t)(hi - lo) * rowb,
+                                cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  }
+  c->release(inv);
+  return MF_OK;
+}
+
 static mf_status init_factors(mf_ctx* c) {
   const size_t es = (size_t)c->ssize();
-  TRY(c->alloc((char**)&c->P, (size_t)c->m * c->k * es));
-  TRY(c->alloc((char**)&c->Q, (size_t)c->n * c->k * es));
   const float amp = (float)std::sqrt(1.0 / ((double)c->k * (double)c->p.init_scale));
   const uint64_t SP = make_stream(c->p.seed, kTagP, 0, 0), SQ = make_stream(c->p.seed, kTagQ, 0, 0);
+  if (c->pq) {
+    TRY(c->alloc((char**)&c->Q, (size_t)c->n * c->k * es));
+    switch (c->p.storage) {
+      case MF_FP32: launch_init<float>(c, c->Q, c->rho_c, c->n, SQ, amp); break;
+      case MF_FP16: launch_init<__half>(c, c->Q, c->rho_c, c->n, SQ, amp); break;
+      default: launch_init<__nv_bfloat16>(c, c->Q, c->rho_c, c->n, SQ, amp); break;
+    }
+    KERNEL_TRY(c);
+    return init_p_out_of_core(c, amp, SP);
+  }
+  TRY(c->alloc((char**)&c->P, (size_t)c->m * c->k * es));
+  TRY(c->alloc((char**)&c->Q, (size_t)c->n * c->k * es));
   switch (c->p.storage) {
     case MF_FP32: launch_init<float>(c, c->P, c->rho_r, c->m, SP, amp);
                   launch_init<float>(c, c->Q, c->rho_c, c->n, SQ, amp); break;
@@ -1193,6 +1292,17 @@ static mf_status setup_staging_buffers(mf_ctx* c) {
     sum += mx;
   }
   cap = std::max<int64_t>(cap, sum);
+  if (c->pq) {                         // one strata block at a time
+    cap = 1;
+    for (size_t b = 0; b + 1 < c->blk_off.size(); ++b) cap = std::max(cap, c->blk_off[b + 1] - c->blk_off[b]);
+    CUDA_TRY(c, cudaStreamCreateWithFlags(&c->ds, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i) {
+      CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_pin[i], cudaEventDisableTiming));
+      CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_pcomp[i], cudaEventDisableTiming));
+      CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_pout[i], cudaEventDisableTiming));
+      CUDA_TRY(c, cudaEventRecord(c->ev_pout[i], c->ds));
+    }
+  }
   c->stg_cap = cap;
   for (int i = 0; i < 2; ++i) {
     TRY(c->alloc(&c->stg[i], (size_t)cap));
@@ -1279,6 +1389,27 @@ static mf_status group_batches(mf_ctx* c, Rating* slots, uint32_t* slot_pos, int
       CUDA_TRY(c, cudaMemcpyAsync(slot_pos + lo, p1, (size_t)n * 4, cudaMemcpyDeviceToDevice, c->st));
   }
   c->release(k0); c->release(k1); c->release(v0); c->release(v1); c->release(tmp); c->release(p1);
+  return MF_OK;
+}
+
+// staged == 2: one strata block's ratings (and duplicate distances) into staging buffer buf,
+// on the copy stream (the caller orders it after the buffer's previous use).
+static mf_status stage_block(mf_ctx* c, int64_t b, int buf) {
+  const int64_t lo = c->blk_off[(size_t)b], len = c->blk_off[(size_t)b + 1] - lo;
+  c->stg_shift[buf].assign(1, {b, -lo});
+  c->stg_len[buf] = len;
+  if (len == 0) return MF_OK;
+  if (c->stg_packed) {
+    CUDA_TRY(c, cudaMemcpyAsync(c->stg_u[buf], c->h_u + lo, (size_t)len * 4, cudaMemcpyHostToDevice, c->cs));
+    CUDA_TRY(c, cudaMemcpyAsync(c->stg_v16[buf], c->h_v16 + lo, (size_t)len * 2, cudaMemcpyHostToDevice, c->cs));
+    CUDA_TRY(c, cudaMemcpyAsync(c->stg_r[buf], c->h_r + lo, (size_t)len * 4, cudaMemcpyHostToDevice, c->cs));
+  } else {
+    CUDA_TRY(c, cudaMemcpyAsync(c->stg[buf], c->h_slots + lo, (size_t)len * sizeof(Rating),
+                                cudaMemcpyHostToDevice, c->cs));
+  }
+  if (c->h_dup)
+    CUDA_TRY(c, cudaMemcpyAsync(c->stg_dup[buf], c->h_dup + lo, (size_t)len * 2, cudaMemcpyHostToDevice, c->cs));
+  c->h2d_bytes += len * (int64_t)((c->stg_packed ? 10 : sizeof(Rating)) + (c->h_dup ? 2 : 0));
   return MF_OK;
 }
 
@@ -1793,6 +1924,33 @@ static mf_status load_test(mf_ctx* c, int64_t N, const int32_t* u, const int32_t
     c->test = kept;
     N = h;
   }
+  if (c->pq && N > 0) {
+    // P out of core: the test ratings grouped by row segment (stable), evaluated one staged
+    // segment at a time
+    Nvtx rg("group test ratings by row segment");
+    uint32_t *k0 = nullptr, *k1 = nullptr, *i0 = nullptr, *i1 = nullptr;
+    unsigned* cnt = nullptr;
+    Rating* sorted = nullptr;
+    TRY(c->alloc(&k0, (size_t)N)); TRY(c->alloc(&k1, (size_t)N));
+    TRY(c->alloc(&i0, (size_t)N)); TRY(c->alloc(&i1, (size_t)N));
+    TRY(c->alloc(&cnt, (size_t)c->a)); TRY(c->alloc(&sorted, (size_t)N));
+    const int g = grid_for(N, c->num_sms);
+    k_test_seg<<<g, 256, 0, c->st>>>(c->test, N, c->m, c->a, k0, i0);
+    KERNEL_TRY(c);
+    TRY(c->sort_pairs(k0, k1, i0, i1, N, bits_for((uint64_t)c->a)));
+    k_gather_records<<<g, 256, 0, c->st>>>(i1, N, nullptr, c->test, nullptr, sorted);
+    CUDA_TRY(c, cudaMemsetAsync(cnt, 0, (size_t)c->a * 4, c->st));
+    k_histogram<<<g, 256, 0, c->st>>>(k1, N, cnt);
+    KERNEL_TRY(c);
+    std::vector<unsigned> hc((size_t)c->a);
+    CUDA_TRY(c, cudaMemcpyAsync(hc.data(), cnt, (size_t)c->a * 4, cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    c->test_seg_off.assign((size_t)c->a + 1, 0);
+    for (int r = 0; r < c->a; ++r) c->test_seg_off[(size_t)r + 1] = c->test_seg_off[(size_t)r] + hc[(size_t)r];
+    c->release(c->test);
+    c->test = sorted;
+    c->release(k0); c->release(k1); c->release(i0); c->release(i1); c->release(cnt);
+  }
   CUDA_TRY(c, cudaStreamSynchronize(c->st));
   c->Ntest = N;
   c->test_loaded = true;
@@ -2160,6 +2318,118 @@ static mf_status prebuild_schedule(mf_ctx* c, int32_t tn) {
   return MF_OK;
 }
 
+// The a sub-epochs of epoch t (A: strata order): Q rotation between them (world > 1), the
+// stratum's ratings staged from host (staged == 1), one interleaved Hogwild launch or one
+// wavefront launch per block.
+static mf_status train_epoch_strata(mf_ctx* c, int32_t t, float g) {
+  // holders of every Q segment's valid copy persist across sub-epochs and epochs (comm);
+  // world == 1 keeps a local vector (every segment is always on rank 0: no transfers)
+  std::vector<int32_t> local_hold((size_t)c->a, -1);
+  int32_t* hold = local_hold.data();
+  std::vector<int32_t> hcopy;
+  if (c->G > 1) {
+    const int32_t* h = c->comm->holders(c->a);
+    hcopy.assign(h, h + c->a);
+    hold = hcopy.data();
+  }
+  std::vector<int64_t> blocks((size_t)c->a), xf((size_t)(5 * c->a));
+  CUDA_TRY(c, cudaEventRecord(c->ev_c0, c->st));
+  CUDA_TRY(c, cudaEventRecord(c->ev_c1, c->st));
+  for (int j = 0; j < c->a; ++j) {
+    Nvtx rj("sub-epoch %d", j);
+    int32_t nb = 0, nx = 0;
+    if (mf_strata_plan(c->p.seed, c->a, c->G, c->rank, c->n, t, j, hold, blocks.data(), &nb,
+                       xf.data(), &nx) != MF_OK)
+      return c->fail(MF_E_INVAL, "strata plan failed");
+    if (nx) {
+      Nvtx rq("Q rotation (%d segments)", nx);
+      TRY(rotate_q(c, xf.data(), nx));
+    }
+    if (c->G > 1) c->comm->set_holders(hold, c->a);
+    int buf = 0;
+    if (c->staged) {
+      // stratum (t, j) is normally pre-staged by the previous step (also across epochs)
+      if (c->staged_t != t || c->staged_j != j) TRY(stage(c, t, j, c->cur_buf));
+      buf = c->cur_buf;
+      const bool last = j + 1 == c->a;
+      TRY(stage(c, last ? t + 1 : t, last ? 0 : j + 1, 1 - buf));   // overlap the next copy
+      CUDA_TRY(c, cudaStreamWaitEvent(c->st, c->ev_h2d[buf], 0));
+      if (c->stg_packed) {
+        if (c->stg_len[buf] > 0) {
+          k_expand_slots<<<grid_for(c->stg_len[buf], c->num_sms), 256, 0, c->st>>>(
+              c->stg_u[buf], c->stg_v16[buf], c->stg_r[buf], c->stg_len[buf], c->stg[buf]);
+          KERNEL_TRY(c);
+          ++c->n_launch;
+        }
+        // the packed buffers are free again once expanded (the slots are stream-ordered);
+        // not so the wavefront's duplicate distances, which the SGD launch reads in place
+        if (!c->h_dup) CUDA_TRY(c, cudaEventRecord(c->ev_free[buf], c->st));
+      }
+    }
+    const int per_launch = (!c->wf && c->p.launch_blocks > 0) ? c->p.launch_blocks : std::max(nb, 1);
+    for (int b0 = 0; b0 < nb; b0 += per_launch)
+      TRY(run_stratum(c, std::vector<int64_t>(blocks.begin() + b0,
+                                              blocks.begin() + std::min(nb, b0 + per_launch)),
+                      g, buf));
+    if (c->staged) {
+      if (!c->stg_packed || c->h_dup) CUDA_TRY(c, cudaEventRecord(c->ev_free[buf], c->st));
+      c->cur_buf = 1 - buf;
+    }
+  }
+  return MF_OK;
+}
+
+// staged == 2 (section 6.1 step 3 + 6.3): blocks one at a time in the strata order, each with
+// its P row segment staged in on the copy stream, trained on the compute stream, written back on
+// the write-back stream; the next block's copy-in overlaps this block's compute, and its
+// write-back the next block's compute.  Two slots: block x uses slot x % 2, which is free once
+// block x-2's write-back is done.  Consecutive blocks of the strata order never share a row
+// segment (a >= 2); every read of a segment is ordered after its last write-back (ds is in
+// order).  Same blocks, same order, same kernels: bit-identical to resident P.
+static mf_status train_epoch_pq(mf_ctx* c, int32_t t, float g) {
+  const size_t rowb = (size_t)c->k * c->ssize();
+  const std::vector<int64_t> pi = host_perm(make_stream(c->p.seed, kTagStrata, (uint64_t)t, 0), c->a);
+  CUDA_TRY(c, cudaEventRecord(c->ev_c0, c->st));
+  CUDA_TRY(c, cudaEventRecord(c->ev_c1, c->st));
+  for (int s = 0; s < 2; ++s) CUDA_TRY(c, cudaStreamWaitEvent(c->cs, c->ev_pout[s], 0));
+  int64_t x = 0;
+  for (int j = 0; j < c->a; ++j) {
+    Nvtx rj("sub-epoch %d", j);
+    for (int r = 0; r < c->a; ++r, ++x) {
+      const int64_t b = (int64_t)r * c->a + (r + pi[(size_t)j]) % c->a;
+      const int s = (int)(x & 1);
+      const int64_t lo = cdiv64((int64_t)r * c->m, c->a), hi = cdiv64((int64_t)(r + 1) * c->m, c->a);
+      const size_t bytes = (size_t)(hi - lo) * rowb;
+      // copy-in
+      CUDA_TRY(c, cudaStreamWaitEvent(c->cs, c->ev_pout[s], 0));
+      TRY(stage_block(c, b, s));
+      CUDA_TRY(c, cudaMemcpyAsync(c->Pslot[s], c->h_P + (size_t)lo * rowb, bytes, cudaMemcpyHostToDevice, c->cs));
+      c->h2d_bytes += (int64_t)bytes;
+      CUDA_TRY(c, cudaEventRecord(c->ev_pin[s], c->cs));
+      // compute
+      CUDA_TRY(c, cudaStreamWaitEvent(c->st, c->ev_pin[s], 0));
+      if (c->stg_packed && c->stg_len[s] > 0) {
+        k_expand_slots<<<grid_for(c->stg_len[s], c->num_sms), 256, 0, c->st>>>(
+            c->stg_u[s], c->stg_v16[s], c->stg_r[s], c->stg_len[s], c->stg[s]);
+        KERNEL_TRY(c);
+        ++c->n_launch;
+      }
+      c->P = c->Pslot[s] - (size_t)lo * rowb;      // P[u] for u in [lo, hi) lands in the slot
+      const mf_status ms = run_stratum(c, std::vector<int64_t>(1, b), g, s);
+      c->P = nullptr;
+      TRY(ms);
+      CUDA_TRY(c, cudaEventRecord(c->ev_pcomp[s], c->st));
+      // write-back
+      CUDA_TRY(c, cudaStreamWaitEvent(c->ds, c->ev_pcomp[s], 0));
+      CUDA_TRY(c, cudaMemcpyAsync(c->h_P + (size_t)lo * rowb, c->Pslot[s], bytes, cudaMemcpyDeviceToHost, c->ds));
+      CUDA_TRY(c, cudaEventRecord(c->ev_pout[s], c->ds));
+    }
+  }
+  // the epoch is complete when its last write-back is
+  CUDA_TRY(c, cudaStreamWaitEvent(c->st, c->ev_pout[(x - 1) & 1], 0));
+  return MF_OK;
+}
+
 mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   if (!c) return MF_E_INVAL;
   TRY(c->enter());
@@ -2224,60 +2494,7 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
     if (epoch_done) *epoch_done = c->t;
     return MF_OK;
   }
-  // holders of every Q segment's valid copy persist across sub-epochs and epochs (comm);
-  // world == 1 keeps a local vector (every segment is always on rank 0: no transfers)
-  std::vector<int32_t> local_hold((size_t)c->a, -1);
-  int32_t* hold = local_hold.data();
-  std::vector<int32_t> hcopy;
-  if (c->G > 1) {
-    const int32_t* h = c->comm->holders(c->a);
-    hcopy.assign(h, h + c->a);
-    hold = hcopy.data();
-  }
-  std::vector<int64_t> blocks((size_t)c->a), xf((size_t)(5 * c->a));
-  CUDA_TRY(c, cudaEventRecord(c->ev_c0, c->st));
-  CUDA_TRY(c, cudaEventRecord(c->ev_c1, c->st));
-  for (int j = 0; j < c->a; ++j) {
-    Nvtx rj("sub-epoch %d", j);
-    int32_t nb = 0, nx = 0;
-    if (mf_strata_plan(c->p.seed, c->a, c->G, c->rank, c->n, t, j, hold, blocks.data(), &nb,
-                       xf.data(), &nx) != MF_OK)
-      return c->fail(MF_E_INVAL, "strata plan failed");
-    if (nx) {
-      Nvtx rq("Q rotation (%d segments)", nx);
-      TRY(rotate_q(c, xf.data(), nx));
-    }
-    if (c->G > 1) c->comm->set_holders(hold, c->a);
-    int buf = 0;
-    if (c->staged) {
-      // stratum (t, j) is normally pre-staged by the previous step (also across epochs)
-      if (c->staged_t != t || c->staged_j != j) TRY(stage(c, t, j, c->cur_buf));
-      buf = c->cur_buf;
-      const bool last = j + 1 == c->a;
-      TRY(stage(c, last ? t + 1 : t, last ? 0 : j + 1, 1 - buf));   // overlap the next copy
-      CUDA_TRY(c, cudaStreamWaitEvent(c->st, c->ev_h2d[buf], 0));
-      if (c->stg_packed) {
-        if (c->stg_len[buf] > 0) {
-          k_expand_slots<<<grid_for(c->stg_len[buf], c->num_sms), 256, 0, c->st>>>(
-              c->stg_u[buf], c->stg_v16[buf], c->stg_r[buf], c->stg_len[buf], c->stg[buf]);
-          KERNEL_TRY(c);
-          ++c->n_launch;
-        }
-        // the packed buffers are free again once expanded (the slots are stream-ordered);
-        // not so the wavefront's duplicate distances, which the SGD launch reads in place
-        if (!c->h_dup) CUDA_TRY(c, cudaEventRecord(c->ev_free[buf], c->st));
-      }
-    }
-    const int per_launch = (!c->wf && c->p.launch_blocks > 0) ? c->p.launch_blocks : std::max(nb, 1);
-    for (int b0 = 0; b0 < nb; b0 += per_launch)
-      TRY(run_stratum(c, std::vector<int64_t>(blocks.begin() + b0,
-                                              blocks.begin() + std::min(nb, b0 + per_launch)),
-                      g, buf));
-    if (c->staged) {
-      if (!c->stg_packed || c->h_dup) CUDA_TRY(c, cudaEventRecord(c->ev_free[buf], c->st));
-      c->cur_buf = 1 - buf;
-    }
-  }
+  TRY(c->pq ? train_epoch_pq(c, t, g) : train_epoch_strata(c, t, g));
   CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
   if (hog) TRY(prebuild_schedule(c, t + 1));   // enqueued after this epoch's SGD launches
   c->t = t + 1;
@@ -2387,6 +2604,33 @@ mf_status mf_rmse(mf_ctx* c, int32_t set, double* out) {
   if (set == MF_TRAIN && (c->G > 1 || c->staged))
     return c->fail(MF_E_UNSUPPORTED, "train-set RMSE needs resident single-GPU ratings");
   Nvtx range("mf_rmse(%s)", set == MF_TRAIN ? "train" : "test");
+  if (c->pq) {
+    // P out of core: one staged row segment at a time (after the epoch's last write-back)
+    CUDA_TRY(c, cudaStreamSynchronize(c->ds));
+    const size_t rowb = (size_t)c->k * c->ssize();
+    double sse = 0.0;
+    for (int r = 0; r < c->a; ++r) {
+      const int64_t t0 = c->test_seg_off.empty() ? 0 : c->test_seg_off[(size_t)r];
+      const int64_t tn = c->test_seg_off.empty() ? 0 : c->test_seg_off[(size_t)r + 1] - t0;
+      if (tn == 0) continue;
+      const int64_t lo = cdiv64((int64_t)r * c->m, c->a), hi = cdiv64((int64_t)(r + 1) * c->m, c->a);
+      CUDA_TRY(c, cudaMemcpyAsync(c->Pslot[0], c->h_P + (size_t)lo * rowb, (size_t)(hi - lo) * rowb,
+                                  cudaMemcpyHostToDevice, c->st));
+      RmseLaunch L{};
+      L.storage = c->p.storage; L.k = c->k; L.test = data + t0; L.N = tn;
+      L.P = c->Pslot[0] - (size_t)lo * rowb; L.Q = c->Q;
+      L.partial = c->rm_partial; L.out = c->rm_out; L.num_sms = c->num_sms; L.stream = c->st;
+      CUDA_TRY(c, launch_rmse(L));
+      double h = 0.0;
+      CUDA_TRY(c, cudaMemcpyAsync(&h, c->rm_out, 8, cudaMemcpyDeviceToHost, c->st));
+      CUDA_TRY(c, cudaStreamSynchronize(c->st));
+      sse += h;
+    }
+    const double rmse = (double)c->p.rating_scale * std::sqrt(sse / std::max((double)N, 1.0));
+    *out = N > 0 ? rmse : 0.0;
+    if (std::isnan(*out)) return c->fail(MF_E_RANGE, "RMSE is NaN (divergence)");
+    return MF_OK;
+  }
   // world > 1: every rank evaluates the test samples of the row segments it owns (filtered at
   // load) against a complete Q, then the SSE and count are summed over ranks.
   if (c->G > 1) TRY(gather_q(c));
@@ -2474,10 +2718,76 @@ static mf_status get_one(mf_ctx* c, const void* X, const int32_t* rho, int64_t r
   return MF_OK;
 }
 
+template <typename X>
+static mf_status d2h(mf_ctx* c, std::vector<X>& h, const X* d, int64_t n) {
+  h.resize((size_t)std::max<int64_t>(n, 1));
+  if (n > 0) CUDA_TRY(c, cudaMemcpyAsync(h.data(), d, (size_t)n * sizeof(X), cudaMemcpyDeviceToHost, c->st));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  return MF_OK;
+}
+
+// staged == 2: P is a host array in relabelled row order and storage type; convert on the host
+// (model_shuffle, Alg. 1 l.15) -- the same values get_one produces on the device.
+template <typename T> static float host_f32(T x);
+template <> float host_f32<float>(float x) { return x; }
+template <> float host_f32<__half>(__half x) { return __half2float(x); }
+template <> float host_f32<__nv_bfloat16>(__nv_bfloat16 x) { return __bfloat162float(x); }
+template <typename T> static T host_from_f32(float x);
+template <> float host_from_f32<float>(float x) { return x; }
+template <> __half host_from_f32<__half>(float x) { return __float2half_rn(x); }
+template <> __nv_bfloat16 host_from_f32<__nv_bfloat16>(float x) { return __float2bfloat16_rn(x); }
+
+template <typename T>
+static void host_p_copy(mf_ctx* c, const std::vector<int32_t>& rho, float* out, const float* in) {
+  const T* X = reinterpret_cast<const T*>(c->h_P);
+  T* Y = reinterpret_cast<T*>(c->h_P);
+  const int64_t k = c->k;
+  for (int64_t id = 0; id < c->m; ++id) {
+    const int64_t row = (int64_t)rho[(size_t)id] * k;
+    for (int64_t d = 0; d < k; ++d) {
+      if (out) out[id * k + d] = host_f32<T>(X[row + d]);
+      else Y[row + d] = host_from_f32<T>(in[id * k + d]);
+    }
+  }
+}
+
+static mf_status pq_p_io(mf_ctx* c, float* out, const float* in, int on_device) {
+  CUDA_TRY(c, cudaStreamSynchronize(c->ds));
+  CUDA_TRY(c, cudaStreamSynchronize(c->st));
+  std::vector<int32_t> rho;
+  TRY(d2h(c, rho, c->rho_r, c->m));
+  const size_t bytes = (size_t)(c->m * c->k) * 4;
+  std::vector<float> stage;
+  float* hout = out;
+  const float* hin = in;
+  if (on_device) {
+    stage.resize((size_t)(c->m * c->k));
+    if (in) {
+      CUDA_TRY(c, cudaMemcpy(stage.data(), in, bytes, cudaMemcpyDeviceToHost));
+      hin = stage.data();
+    } else {
+      hout = stage.data();
+    }
+  }
+  switch (c->p.storage) {
+    case MF_FP32: host_p_copy<float>(c, rho, hout, hin); break;
+    case MF_FP16: host_p_copy<__half>(c, rho, hout, hin); break;
+    default: host_p_copy<__nv_bfloat16>(c, rho, hout, hin); break;
+  }
+  if (on_device && out) CUDA_TRY(c, cudaMemcpy(out, stage.data(), bytes, cudaMemcpyHostToDevice));
+  return MF_OK;
+}
+
 mf_status mf_get_factors(mf_ctx* c, float* P, float* Q, int32_t on_device) {
   if (!c) return MF_E_INVAL;
   TRY(c->enter());
   if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
+  if (c->pq) {
+    if (P) TRY(pq_p_io(c, P, nullptr, on_device));
+    if (Q) TRY(get_one(c, c->Q, c->rho_c, c->n, Q, on_device));
+    CUDA_TRY(c, cudaStreamSynchronize(c->st));
+    return MF_OK;
+  }
   if (c->G > 1) {
     TRY(gather_q(c));
     std::string why;
@@ -2517,6 +2827,10 @@ mf_status mf_set_factors(mf_ctx* c, const float* P, const float* Q, int32_t on_d
   if (!c) return MF_E_INVAL;
   TRY(c->enter());
   if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
+  if (c->pq && P) {
+    TRY(pq_p_io(c, nullptr, P, on_device));
+    P = nullptr;
+  }
   if (P) TRY(set_one(c, c->P, c->rho_r, c->m, P, on_device));
   if (Q) TRY(set_one(c, c->Q, c->rho_c, c->n, Q, on_device));
   if (c->G > 1 && Q) c->comm->reset_holders(c->a);  // every rank holds a valid copy again
@@ -2538,13 +2852,6 @@ mf_status mf_get_epoch(const mf_ctx* c, int32_t* t) {
 // ---------------------------------------------------------------------------------------------
 // exports
 // ---------------------------------------------------------------------------------------------
-template <typename X>
-static mf_status d2h(mf_ctx* c, std::vector<X>& h, const X* d, int64_t n) {
-  h.resize((size_t)std::max<int64_t>(n, 1));
-  if (n > 0) CUDA_TRY(c, cudaMemcpyAsync(h.data(), d, (size_t)n * sizeof(X), cudaMemcpyDeviceToHost, c->st));
-  CUDA_TRY(c, cudaStreamSynchronize(c->st));
-  return MF_OK;
-}
 
 mf_status mf_export_schedule(mf_ctx* c, int32_t what, int32_t epoch, int64_t* buf, int64_t* len) {
   if (!c || !len) return MF_E_INVAL;

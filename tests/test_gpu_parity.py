@@ -641,6 +641,46 @@ def test_out_of_core_load_below_the_device_budget_is_bit_identical(kw):
     assert np.array_equal(P0, P1) and np.array_equal(Q0, Q1) and r0 == r1
 
 
+@pytest.mark.parametrize("kw", [dict(schedule="hogwild", workers=1, grid_a=8, batch_f=256),
+                                dict(schedule="wavefront", workers=4, wf_cols=6, grid_a=8, storage="fp16"),
+                                dict(schedule="hogwild", workers=1, grid_a=16, batch_f=64, storage="bf16")])
+def test_p_out_of_core_below_the_device_budget_is_bit_identical(kw):
+    """Section 6.1 step 3 / 6.3 (staged = 2): P larger than the device budget too.  P's row
+    segments live in pinned host memory; every strata block runs with its segment copied in
+    (copy stream), trained, and written back (D2H stream) while the next block computes; Q stays
+    resident; the two segment slots take 2/a of P.  Under a device budget below P alone
+    (a = 8, 16), the trained P and Q are bit-identical to the resident run (the test RMSE,
+    evaluated segment by segment, to 1e-12); set_factors / get_factors go through the host
+    copy."""
+    R = synth.uniform(m=200_000, n=2000, N=1_000_000, seed=4, mu=0.5, rank=4, noise=0.1, Ntest=20_000)
+    k = 64
+    p_bytes = R.m * k * (4 if kw.get("storage", "fp32") == "fp32" else 2)
+    out = []
+    for staged in (0, 2):
+        extra = dict(staged=2, stage_chunk=1 << 17, device_budget=p_bytes * 3 // 4) if staged else {}
+        g = mf.MF(R.m, R.n, k, **TABLE3_NETFLIX, **kw, **extra)
+        g.load(R.u, R.v, R.r)
+        g.load(R.ut, R.vt, R.rt, "test")
+        r0 = g.rmse()
+        for _ in range(2):
+            g.train_epoch()
+            assert g.stats()["updates"] == R.N
+        assert g.check_visits()["bad_units"] == 0
+        if staged:
+            assert 0 < g.device_peak_bytes < p_bytes, (g.device_peak_bytes, p_bytes)
+        out.append((g.factors(), g.rmse(), r0))
+        if staged:          # host-side set/get round trip of P (rounded to storage)
+            P, Q = out[-1][0]
+            g.set_factors(P=P)
+            assert np.array_equal(g.factors()[0], P)
+        g.close()
+    (P0, Q0), r0, i0 = out[0]
+    (P1, Q1), r1, i1 = out[1]
+    assert np.array_equal(P0, P1) and np.array_equal(Q0, Q1)
+    # the segment-by-segment RMSE sums the same squared errors in another order
+    assert abs(i0 - i1) <= 1e-12 * i0 and abs(r0 - r1) <= 1e-12 * r0, (i0, i1, r0, r1)
+
+
 def test_resident_load_fails_cleanly_below_the_device_budget():
     """The same budget without out-of-core staging: the resident preprocessing needs the whole
     set in HBM, so the load fails with MF_E_NOMEM (and the ctx stays usable)."""
