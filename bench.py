@@ -60,8 +60,9 @@ def parse():
                     help="batch-Hogwild with column-grouped batches (reading R24, params.group_cols)")
     ap.add_argument("--exact-order", action="store_true",
                     help="evaluate Alg. 1 l.8-10 in the paper's operation order (params.exact_order)")
-    ap.add_argument("--staged", action="store_true",
-                    help="out-of-core: ratings in pinned host memory, streamed per stratum")
+    ap.add_argument("--staged", type=int, nargs="?", const=1, default=0,
+                    help="out-of-core: 1 = ratings in pinned host memory, streamed per stratum; "
+                         "2 = P's row segments too, one strata block at a time")
     ap.add_argument("--grid-a", type=int, default=0)
     ap.add_argument("--lr-rule", default="eq9", choices=["eq9", "adagrad"])
     ap.add_argument("--batch-f", type=int, default=0, help="Eq. 8 f (0 = 256, P:L277)")
@@ -326,7 +327,7 @@ def config_of(args, R, world):
             "fraction": args.fraction, "exact_order": bool(args.exact_order),
             "rating_stage": "tma" if args.rating_stage else "lane-loads",
             "group_cols": bool(args.group_cols),
-            "staged": bool(args.staged), "grid_a": args.grid_a or (8 if world > 1 else 1),
+            "staged": int(args.staged), "grid_a": args.grid_a or (8 if world > 1 else 1),
             "l2": "inputs larger than L2 (COO %.2f GB per epoch); model P+Q stays cached as in "
                   "any training run" % (R.N * 12 / 1e9)}
 
@@ -558,7 +559,7 @@ def run_e2e(args, R, kw, stream, C):
     from paper_conf_hpdc_xietfl17_b200 import mf
     world = C.world
     kw2 = dict(kw)
-    kw2["staged"] = True
+    kw2["staged"] = max(1, int(args.staged))
     host = None
     if world == 1:
         host = [x.cpu().pin_memory().numpy() for x in (R.u, R.v, R.r, R.ut, R.vt, R.rt)]

@@ -34,6 +34,7 @@ ap.add_argument("--out", default=None)
 ap.add_argument("--gs", default="1,2,4,8", help="GPU counts to emulate")
 ap.add_argument("--workers", default="0", help="comma list of Hogwild worker counts (0 = all resident)")
 ap.add_argument("--no-base", action="store_true")
+ap.add_argument("--group-cols", action="store_true", help="column-grouped batches (R24) in the G runs")
 args = ap.parse_args()
 
 s = synth.SHAPES[args.workload]
@@ -70,13 +71,15 @@ if not args.no_base:
     rows.append(dict(G=1, grid="a=1 f=256", ms_epoch=t1, gups=upd / t1 / 1e6, rmse=rmse1))
     print(json.dumps(rows[-1]), flush=True)
 for G, W in [(int(g), int(w)) for g in args.gs.split(",") for w in args.workers.split(",")]:
-    per, rmse, upd = run(grid_a=A, batch_f=args.batch_f, launch_blocks=A // G, workers=W)
+    per, rmse, upd = run(grid_a=A, batch_f=args.batch_f, launch_blocks=A // G, workers=W,
+                         group_cols=args.group_cols)
     assert per.shape[1] == A * G, per.shape
     t = per.reshape(per.shape[0], A, G)                     # [epoch, sub-epoch j, rank g]
     comp = float(t.max(2).sum(1).mean())
     imb = float((t.max(2) / t.mean(2)).mean())
     tg = comp + (A * t_comm if G > 1 else 0.0)
-    rows.append(dict(G=G, workers=W, grid=f"a={A} f={args.batch_f} blocks/launch={A // G}",
+    rows.append(dict(G=G, workers=W, grid=f"a={A} f={args.batch_f} blocks/launch={A // G}"
+                     + (" grouped" if args.group_cols else ""),
                      compute_ms=comp, comm_ms_est=A * t_comm if G > 1 else 0.0, ms_epoch=tg,
                      gups=upd / tg / 1e6, per_gpu_gups=upd / tg / 1e6 / G,
                      efficiency_vs_a1=(upd / tg) / (G * upd / t1), load_imbalance=imb, rmse=rmse))
