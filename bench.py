@@ -58,6 +58,8 @@ def parse():
                     help="Hogwild rating stream: 0 = per-lane loads, 1 = TMA bulk copies")
     ap.add_argument("--group-cols", action="store_true",
                     help="batch-Hogwild with column-grouped batches (reading R24, params.group_cols)")
+    ap.add_argument("--plain-batches", action="store_true",
+                    help="N > 1: keep the storage order inside batches (no column grouping)")
     ap.add_argument("--exact-order", action="store_true",
                     help="evaluate Alg. 1 l.8-10 in the paper's operation order (params.exact_order)")
     ap.add_argument("--staged", type=int, nargs="?", const=1, default=0,
@@ -278,11 +280,25 @@ def default_f(args, world):
     """Eq. 8 batch f (256).  N > 1 on the Yahoo shape: f = 64 -- each rank's sub-epoch
     launch holds ~1/64 of the ratings, so 256-sample chunks would leave ~1.6 chunks per worker
     and a quantised tail (emulated G = 8: 49.3 -> 54.3 G updates/s, same RMSE;
-    profiles/r01_scaling_hot_rows.md section 6).  Hugewiki's launches hold ~20 chunks of 256
-    per worker even at G = 8."""
+    profiles/r01_scaling_hot_rows.md section 6).  Column-grouped batches (the N > 1 default on
+    the power-law shapes, R24): f = 1024 (profiles/r02_scaling.md)."""
     if args.batch_f:
         return args.batch_f
+    if args.group_cols:
+        return 1024
     return 64 if (world > 1 and args.workload == "yahoo") else 256
+
+
+def resolve_group(args, world):
+    """N > 1 on the Hugewiki / Netflix shapes: column-grouped batches (R24) by default.  A DSGD
+    strata block sees only n/a columns, so a power-law-hot column takes an a-fold larger share
+    of its block's updates and Hogwild runs at that column's read-modify-write rate; grouping
+    keeps a batch's run of the column in registers.  Emulated Hugewiki (half size) at G = 8:
+    10.0 -> 23.4 G updates/s, load imbalance 1.34 -> 1.07 (profiles/r02_scaling.md).
+    --plain-batches keeps the paper's storage order inside batches."""
+    if world > 1 and args.workload in ("hugewiki", "netflix") and not args.plain_batches \
+            and args.schedule == "hogwild":
+        args.group_cols = True
 
 
 def run_reference(args):
@@ -617,6 +633,7 @@ def main():
     if args.emulate_ranks > 1:
         world = args.emulate_ranks
         resolve_workload(args, world)
+        resolve_group(args, world)
         torch.cuda.set_device(0)
         R = workload(args, torch.device("cuda:0"))
         group = ThreadGroup(world)
@@ -640,6 +657,7 @@ def main():
         return
     C = DistRanks()
     resolve_workload(args, C.world)
+    resolve_group(args, C.world)
     line = rank_main(args, C)
     if line is not None:
         print(json.dumps(line), flush=True)

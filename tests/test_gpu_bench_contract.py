@@ -63,6 +63,7 @@ def test_bench_multirank_path_emulated(ranks):
     assert d["n_gpus"] == ranks and d["scaling"] == "strong"
     assert d["config"]["workload"].startswith("hugewiki") and d["config"]["grid_a"] == 8
     assert d["config"]["parallelism"] == f"dsgd-strata{ranks}"
+    assert d["config"]["group_cols"] is True and d["config"]["batch_f"] == 1024
     eo = d["exactly_once"]
     assert eo["bad_units"] == 0 and eo["updates_per_epoch"] == eo["N"] == d["config"]["N_train"]
     assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0

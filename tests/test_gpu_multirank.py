@@ -57,7 +57,8 @@ def run_ranks(world, R, k, epochs, **kw):
 @pytest.mark.parametrize("world", [2, 4])
 @pytest.mark.parametrize("kw", [dict(schedule="wavefront", workers=4, wf_cols=5),
                                 dict(schedule="hogwild", workers=1, batch_f=64),
-                                dict(schedule="wavefront", workers=4, wf_cols=5, staged=True)])
+                                dict(schedule="wavefront", workers=4, wf_cols=5, staged=True),
+                                dict(schedule="hogwild", workers=1, batch_f=64, group_cols=True)])
 def test_multirank_strata_matches_oracle(world, kw):
     R = synth.tiny(seed=0)
     epochs = 2
