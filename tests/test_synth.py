@@ -69,3 +69,25 @@ def test_cuda_rendering_is_bit_identical_to_cpu():
         g = synth.shaped(name, fraction=frac, device="cuda")
         assert synth.checksum(c) == synth.checksum(g), name
         assert torch.equal(c.r, g.r.cpu()) and torch.equal(c.v, g.v.cpu()), name
+
+
+def test_table2_shapes_and_table3_hyperparameters():
+    """Table 2 shapes and Table 3 hyper-parameters of the configs."""
+    want = {"netflix": (480_190, 17_771, 99_072_112, 1_408_395, 0.05, 0.08, 0.3),
+            "yahoo": (1_000_990, 624_961, 252_800_275, 4_003_960, 1.0, 0.08, 0.2),
+            "hugewiki": (50_082_604, 39_781, 3_069_817_980, 31_327_899, 0.03, 0.08, 0.3)}
+    for name, (m, n, N, Nt, lam, alpha, beta) in want.items():
+        s = synth.SHAPES[name]
+        assert (s["m"], s["n"], s["N"], s["Ntest"]) == (m, n, N, Nt), name
+        assert (s["lam"], s["alpha"], s["beta"]) == (lam, alpha, beta), name
+    R = synth.shaped("yahoo", fraction=0.0005)
+    assert (R.m, R.n, R.N, R.Ntest) == (500, 312, 126_400, 2_001)
+    assert 0.0 <= float(R.r.min()) and float(R.r.max()) <= 100.0      # Yahoo's 0-100 scale
+
+
+def test_eq5_byte_and_flop_accounting():
+    """Eq. 5: one update at k = 128 with fp32 features moves 12 + 4 k 4 = 2060 bytes
+    for 7k - 1 = 895 flops, 0.43 flop/B -- the algorithmic bytes bench.py divides by (fp16: 1036)."""
+    k = 128
+    assert 12 + 4 * k * 4 == 2060 and 12 + 4 * k * 2 == 1036
+    assert 7 * k - 1 == 895 and round(895 / 2060, 2) == 0.43
