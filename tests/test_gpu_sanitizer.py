@@ -33,10 +33,17 @@ def _run(tool, which, timeout=900):
 
 def test_memcheck_all_kernels():
     out = _run("memcheck", "all")
-    assert out.count("ok {") == 11
+    assert out.count("ok {") == 18
 
 
 @pytest.mark.parametrize("tool", ["racecheck", "synccheck"])
 def test_deterministic_kernels_race_and_sync_clean(tool):
     out = _run(tool, "det")
-    assert out.count("ok {") == 6
+    assert out.count("ok {") == 8
+
+
+def test_tma_rating_ring_race_clean():
+    """The TMA rating stream's shared-memory ring (bulk copies, mbarriers, generic reads) under
+    racecheck, at 1 worker (no by-design races on P/Q)."""
+    out = _run("racecheck", "smem")
+    assert out.count("ok {") == 2

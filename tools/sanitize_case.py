@@ -23,6 +23,10 @@ DET = [
     dict(k=16, storage="fp32", schedule="wavefront", workers=4, wf_cols=8),                 # 16-lane ring
     dict(k=32, storage="fp32", schedule="wavefront", workers=4, wf_cols=8, wf_kernel=2),    # register
     dict(k=32, storage="fp32", schedule="wavefront", workers=4, wf_cols=8, lr_rule="adagrad"),
+    dict(k=128, storage="fp16", schedule="wavefront", workers=6, wf_cols=9, exact_order=True,
+         check_owners=True),                                                                # exact form + checker
+    dict(k=64, storage="fp32", schedule="wavefront", workers=4, wf_cols=6, grid_a=4, staged=2,
+         stage_chunk=1000),                                                                 # P out of core
 ]
 RACY = [
     dict(k=16, storage="fp32", schedule="hogwild"),
@@ -30,6 +34,12 @@ RACY = [
     dict(k=128, storage="bf16", schedule="hogwild", staged=True, grid_a=2),
     dict(k=64, storage="fp32", schedule="libmf", grid_a=4),
     dict(k=32, storage="fp32", schedule="hogwild", lr_rule="adagrad"),
+    dict(k=128, storage="fp16", schedule="hogwild", rating_stage=1, batch_f=128),      # TMA rating stream
+    dict(k=128, storage="fp16", schedule="hogwild", group_cols=True, batch_f=512),     # grouped batches
+    dict(k=32, storage="fp32", schedule="hogwild", grid_a=4, batch_f=64, staged=True,
+         stage_chunk=1500),                                                             # chunked out-of-core load
+    dict(k=128, storage="bf16", schedule="hogwild", grid_a=4, batch_f=64, staged=2),   # P out of core
+    dict(k=16, storage="fp16", schedule="hogwild", exact_order=True),
 ]
 
 
@@ -57,7 +67,15 @@ def run(case):
     print("ok", case, round(rm, 5), flush=True)
 
 
+# shared-memory rings of the Hogwild kernels (TMA rating stream), at 1 worker so that the global
+# P/Q accesses do not race by design either: racecheck then checks the smem ring protocol
+SMEM = [
+    dict(k=128, storage="fp16", schedule="hogwild", rating_stage=1, batch_f=128, workers=1),
+    dict(k=64, storage="fp32", schedule="hogwild", rating_stage=1, batch_f=64, workers=1, grid_a=2),
+]
+
 if __name__ == "__main__":
     which = sys.argv[1] if len(sys.argv) > 1 else "all"
-    for c in DET + (RACY if which == "all" else []):
+    cases = {"all": DET + RACY, "det": DET, "smem": SMEM}[which]
+    for c in cases:
         run(c)
