@@ -85,7 +85,8 @@ typedef struct mf_params {
   int32_t schedule;       /* mf_schedule                                                        */
   int32_t storage;        /* mf_storage of P and Q; arithmetic is always fp32                   */
   int32_t workers;        /* s: Hogwild = concurrent sample groups (0 = all resident);
-                             wavefront = row sub-blocks per strata block (0 = min(768, m/(4a)))             */
+                             wavefront = row sub-blocks per strata block (0 = min(768/(a/world),
+                             m/(4a)): one launch runs the a/world blocks of a stratum together) */
   int32_t batch_f;        /* Eq. 8 batch f (0 = 256)                                    */
   int32_t wf_cols;        /* wavefront column sub-blocks c (0 = 2*s, R9)                        */
   int32_t grid_a;         /* strata grid a x a (0 = 1 if world == 1 else 8); a % world == 0

@@ -976,7 +976,11 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   c->pq = p->staged == 2;
   if (c->wf) {
     const int64_t rows_per_seg = p->m / a;
-    int64_t s = p->workers > 0 ? p->workers : std::min<int64_t>(768, std::max<int64_t>(1, rows_per_seg / 4));
+    // default s: 768 workers per launch (all co-resident in every ring geometry), shared by the
+    // a / G blocks of a stratum that one launch runs together
+    const int64_t cap = std::max<int64_t>(1, 768 / std::max(1, a / world));
+    int64_t s = p->workers > 0 ? p->workers
+                               : std::min<int64_t>(cap, std::max<int64_t>(1, rows_per_seg / 4));
     c->s = (int)s;
     c->c = p->wf_cols > 0 ? p->wf_cols : 2 * c->s;
     if (p->cyclic && c->c < c->s) { delete c; return MF_E_INVAL; }
@@ -1217,11 +1221,12 @@ static mf_status alloc_schedule(mf_ctx* c) {
   if (c->wf) {
     TRY(c->alloc(&c->seq, (size_t)cap));
     TRY(c->alloc(&c->rank_arr, (size_t)cap));
-    TRY(c->alloc(&c->tickets, (size_t)c->c));
+    const size_t per_launch = (size_t)(c->a / c->G) * c->c;   // c per block of a stratum
+    TRY(c->alloc(&c->tickets, per_launch));
     if (c->p.check_owners) {
-      TRY(c->alloc(&c->owners, (size_t)c->c));
+      TRY(c->alloc(&c->owners, per_launch));
       TRY(c->alloc(&c->own_viol, 1));
-      CUDA_TRY(c, cudaMemsetAsync(c->owners, 0xFF, (size_t)c->c * 4, c->st));   // all free (-1)
+      CUDA_TRY(c, cudaMemsetAsync(c->owners, 0xFF, per_launch * 4, c->st));   // all free (-1)
       CUDA_TRY(c, cudaMemsetAsync(c->own_viol, 0, 4, c->st));
     }
     if (c->p.cyclic) {
@@ -2176,46 +2181,67 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     ++c->n_launch;
     return MF_OK;
   }
-  for (int64_t b : blocks) {
-    if (c->blk_len[(size_t)b] == 0) continue;
-    CUDA_TRY(c, cudaMemsetAsync(c->tickets, 0, (size_t)c->c * 4, c->st));
-    const int64_t base = b * (int64_t)c->s * c->c;
+  // The non-empty blocks run together in one cooperative launch (they touch disjoint rows and
+  // columns, so any concurrency gives the result of running them one after another): worker w
+  // of the launch is worker w % s of block w / s, with c tickets per block.  When s x blocks
+  // workers cannot all be co-resident, the blocks go in smaller groups (down to one per launch).
+  std::vector<int64_t> todo;
+  for (int64_t b : blocks)
+    if (c->blk_len[(size_t)b] > 0) todo.push_back(b);
+  size_t group = std::max<size_t>(todo.size(), 1);
+  static const bool kProfWaves = std::getenv("MF_PROFILE_WAVES") != nullptr;
+  for (size_t g0 = 0; g0 < todo.size();) {
+    const size_t gn = std::min(group, todo.size() - g0);
     WavefrontLaunch L{};
-    L.storage = c->p.storage; L.k = c->k; L.slots = slots; L.sub_off = c->sub_off + base;
-    L.shift = slot_shift(c, buf, b);
+    L.blocks.n = (int)gn;
+    for (size_t i = 0; i < gn; ++i) {
+      const int64_t b = todo[g0 + i];
+      L.blocks.base[i] = b * (int64_t)c->s * c->c;
+      L.blocks.shift[i] = slot_shift(c, buf, b);
+    }
+    CUDA_TRY(c, cudaMemsetAsync(c->tickets, 0, gn * (size_t)c->c * 4, c->st));
+    L.storage = c->p.storage; L.k = c->k; L.slots = slots; L.sub_off = c->sub_off;
     L.variant = c->p.wf_kernel == 2 ? 0 : 1;
     L.lane_bytes = c->p.lane_bytes;
     L.dup = dup;
-    L.seq = c->seq + base; L.rank = c->rank_arr + base; L.tickets = c->tickets;
+    L.seq = c->seq; L.rank = c->rank_arr; L.tickets = c->tickets;
     L.s = c->s; L.c = c->c; L.num_sms = c->num_sms; L.P = c->P; L.Q = c->Q; L.g = g;
     L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
     L.ada = ada_args(c);
     L.exact = c->p.exact_order;
     if (L.ada.GP) L.g = c->p.alpha;
     L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
-    L.visits = c->visits + base; L.upd = c->upd_dev;
+    L.visits = c->visits; L.upd = c->upd_dev;
     L.owners = c->owners; L.viol = c->own_viol;
     // Diagnostics only (MF_PROFILE_WAVES=1): per-worker clock64 totals of ticket waits and
     // sub-block runs, summarised on stderr after the launch (synchronises).
-    static const bool kProfWaves = std::getenv("MF_PROFILE_WAVES") != nullptr;
+    const int nw = c->s * (int)gn;
     long long* prof = nullptr;
     if (kProfWaves && L.variant == 1) {
-      CUDA_TRY(c, cudaMallocAsync(reinterpret_cast<void**>(&prof), (size_t)c->s * 6 * 8, c->st));
-      CUDA_TRY(c, cudaMemsetAsync(prof, 0, (size_t)c->s * 6 * 8, c->st));
+      CUDA_TRY(c, cudaMallocAsync(reinterpret_cast<void**>(&prof), (size_t)nw * 6 * 8, c->st));
+      CUDA_TRY(c, cudaMemsetAsync(prof, 0, (size_t)nw * 6 * 8, c->st));
     }
     L.prof = prof;
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
     cudaError_t e = launch_wavefront(L);
+    if (e == cudaErrorCooperativeLaunchTooLarge) {
+      cudaGetLastError();
+      if (prof) CUDA_TRY(c, cudaFreeAsync(prof, c->st));
+      if (gn == 1)
+        return c->fail(MF_E_UNSUPPORTED, "wavefront: %d workers cannot all be co-resident", c->s);
+      group = std::max<size_t>(1, gn / 2);                  // retry with smaller groups
+      continue;
+    }
     if (prof && e == cudaSuccess) {
-      std::vector<long long> h((size_t)c->s * 6);
+      std::vector<long long> h((size_t)nw * 6);
       CUDA_TRY(c, cudaMemcpyAsync(h.data(), prof, h.size() * 8, cudaMemcpyDeviceToHost, c->st));
       CUDA_TRY(c, cudaStreamSynchronize(c->st));
       CUDA_TRY(c, cudaFreeAsync(prof, c->st));
       std::map<long long, int> per_smsp;
-      for (int i = 0; i < c->s; ++i) ++per_smsp[h[6 * i + 3] * 4 + (h[6 * i + 4] & 3)];
+      for (int i = 0; i < nw; ++i) ++per_smsp[h[6 * i + 3] * 4 + (h[6 * i + 4] & 3)];
       double sw = 0, sr = 0, mxw = 0, mxr = 0, mxt = 0, sn = 0, shared_r = 0, solo_r = 0;
       double shared_n = 0, solo_n = 0, srel = 0;
-      for (int i = 0; i < c->s; ++i) {
+      for (int i = 0; i < nw; ++i) {
         const double w = (double)h[6 * i], r = (double)h[6 * i + 1], n = (double)h[6 * i + 2];
         srel += (double)h[6 * i + 5];
         sw += w; sr += r; sn += n;
@@ -2227,23 +2253,20 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
       int shared_w = 0;
       for (auto& kv : per_smsp) if (kv.second > 1) shared_w += kv.second;
       std::fprintf(stderr,
-                   "[MF_PROFILE_WAVES] s=%d c=%d  cycles/worker: wait mean %.3g max %.3g, run mean %.3g "
-                   "max %.3g, wait+run max %.3g; run cycles/sample %.1f (solo-SMSP workers %.1f, "
+                   "[MF_PROFILE_WAVES] s=%d c=%d blocks=%d  cycles/worker: wait mean %.3g max %.3g, run mean "
+                   "%.3g max %.3g, wait+run max %.3g; run cycles/sample %.1f (solo-SMSP workers %.1f, "
                    "SMSP-sharing %.1f; %d of %d workers share an SMSP); release fence mean %.3g cycles/worker\n",
-                   c->s, c->c, sw / c->s, mxw, sr / c->s, mxr, mxt, sr / std::max(sn, 1.0),
-                   solo_r / std::max(solo_n, 1.0), shared_r / std::max(shared_n, 1.0), shared_w, c->s,
-                   srel / c->s);
-    }
-    if (e == cudaErrorCooperativeLaunchTooLarge) {
-      cudaGetLastError();
-      return c->fail(MF_E_UNSUPPORTED, "wavefront: %d workers cannot all be co-resident", c->s);
+                   c->s, c->c, (int)gn, sw / nw, mxw, sr / nw, mxr, mxt, sr / std::max(sn, 1.0),
+                   solo_r / std::max(solo_n, 1.0), shared_r / std::max(shared_n, 1.0), shared_w, nw,
+                   srel / nw);
     }
     CUDA_TRY(c, e);
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd + 1), c->st));
-    c->last_workers = c->s;
+    c->last_workers = nw;
     c->last_block = 128;
     ++c->n_sgd;
     ++c->n_launch;
+    g0 += gn;
   }
   return MF_OK;
 }

@@ -49,11 +49,19 @@ struct HogwildLaunch {
   int *out_workers, *out_lanes, *out_grid;
 };
 
+// The strata blocks one wavefront launch runs concurrently (a stratum's blocks touch disjoint
+// rows and columns): worker w of the launch is worker w % s of block w / s.
+struct WfBlocks {
+  int n;
+  int64_t base[kMaxSegs];   // b * s * c: offset of the block's sub_off / seq / rank / visits
+  int64_t shift[kMaxSegs];  // slot shift of the block (0 resident; staged: buffer offset - start)
+};
+
 struct WavefrontLaunch {
   int storage, k, variant;  // variant 1 = ring-staged k_wavefront2 (needs dup), 0 = k_wavefront
   int lane_bytes;           // ring kernel: 16 (default) or 32 bytes per lane
   const Rating* slots;
-  int64_t shift;           // slot index offset (0 resident; staged: buffer offset - block start)
+  WfBlocks blocks;          // the blocks of this launch (tickets / owners: c per block, in order)
   const uint16_t* dup;     // per slot: distance to previous same-u (low byte) / same-v (high
                            // byte) sample of the sub-block if <= ring_window(), else 0
   const int64_t* sub_off;  // s*c + 1 slot offsets of this strata block's sub-blocks

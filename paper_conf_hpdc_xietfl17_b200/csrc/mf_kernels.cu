@@ -158,7 +158,7 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
                                                    const int32_t* __restrict__ rank,
                                                    int* __restrict__ tickets, int s, int c,
                                                    T* __restrict__ P, T* __restrict__ Q, Step st,
-                                                   int64_t shift, AdaArgs ada,
+                                                   WfBlocks bl, AdaArgs ada,
                                                    unsigned* __restrict__ visits,
                                                    unsigned long long* __restrict__ upd,
                                                    int* __restrict__ owners,
@@ -166,8 +166,16 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
   const int lane = threadIdx.x & 31;
   const int grp = lane / L, gl = lane % L, gbase = grp * L;
   const unsigned gmask = (L == 32) ? 0xffffffffu : (((1u << L) - 1u) << gbase);
-  const int worker = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) / L);
-  if (worker >= s) return;
+  const int gw = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) / L);
+  if (gw >= s * bl.n) return;
+  const int bi = gw / s, worker = gw - bi * s;      // block of the launch, worker in the block
+  const int64_t shift = bl.shift[bi];
+  sub_off += bl.base[bi];
+  seq += bl.base[bi];
+  rank += bl.base[bi];
+  visits += bl.base[bi];
+  tickets += (int64_t)bi * c;
+  if (owners) owners += (int64_t)bi * c;
   const int32_t* my_seq = seq + (int64_t)worker * c;
   const int32_t* my_rank = rank + (int64_t)worker * c;
   int done = 0;
@@ -198,7 +206,7 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
                                                     const int32_t* __restrict__ rank,
                                                     int* __restrict__ tickets, int s, int c,
                                                     T* __restrict__ P, T* __restrict__ Q, Step st,
-                                                    int64_t shift,
+                                                    WfBlocks bl,
                                                     long long* __restrict__ prof,
                                                     unsigned* __restrict__ visits,
                                                     unsigned long long* __restrict__ upd,
@@ -213,8 +221,16 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
   // spins on its own ticket) and serialise each other's instruction streams
   if (lane >= L) return;
   const int local = threadIdx.x >> 5;
-  const int worker = blockIdx.x * (blockDim.x >> 5) + local;
-  if (worker >= s) return;
+  const int gw = blockIdx.x * (blockDim.x >> 5) + local;
+  if (gw >= s * bl.n) return;
+  const int bi = gw / s, worker = gw - bi * s;      // block of the launch, worker in the block
+  const int64_t shift = bl.shift[bi];
+  sub_off += bl.base[bi];
+  seq += bl.base[bi];
+  rank += bl.base[bi];
+  visits += bl.base[bi];
+  tickets += (int64_t)bi * c;
+  if (owners) owners += (int64_t)bi * c;
   char* ring = smem + (size_t)local * RS * 2 * ROWB;
   const int32_t* my_seq = seq + (int64_t)worker * c;
   const int32_t* my_rank = rank + (int64_t)worker * c;
@@ -301,7 +317,7 @@ __global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ s
     unsigned smid, wid;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
     asm volatile("mov.u32 %0, %%warpid;" : "=r"(wid));
-    long long* o = prof + 6 * (int64_t)worker;
+    long long* o = prof + 6 * (int64_t)gw;
     o[0] = t_wait; o[1] = t_run; o[2] = n_done; o[3] = smid; o[4] = wid; o[5] = t_rel;
   }
 }
@@ -534,7 +550,7 @@ template <typename T, int K, int L, bool ADA = false, bool EX = false>
 static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
   auto kern = k_wavefront<T, K, L, ADA, EX>;
   const int threads = 128;
-  const int64_t total_threads = (int64_t)a.s * L;
+  const int64_t total_threads = (int64_t)a.s * a.blocks.n * L;
   const int blocks = (int)cdiv64(total_threads, threads);
   int per_sm = 0;
   cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, 0);
@@ -551,13 +567,13 @@ static cudaError_t launch_wavefront_t(const WavefrontLaunch& a) {
   T* P = reinterpret_cast<T*>(a.P);
   T* Q = reinterpret_cast<T*>(a.Q);
   Step st = step_of(a);
-  int64_t shift = a.shift;
+  WfBlocks bl = a.blocks;
   AdaArgs ada = a.ada;
   unsigned* visits = a.visits;
   unsigned long long* upd = a.upd;
   int* owners = a.owners;
   unsigned* viol = a.viol;
-  void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &st, &shift,
+  void* args[] = {&slots, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &st, &bl,
                   &ada, &visits, &upd, &owners, &viol};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, 0,
                                      a.stream);
@@ -576,7 +592,7 @@ static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
   const size_t smem = (size_t)wpc * RS * 2 * ROWB;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  const int blocks = (int)cdiv64((int64_t)a.s, wpc);
+  const int blocks = (int)cdiv64((int64_t)a.s * a.blocks.n, wpc);
   int per_sm = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, smem);
   if (e != cudaSuccess) return e;
@@ -593,14 +609,14 @@ static cudaError_t launch_wavefront2_t(const WavefrontLaunch& a) {
   T* P = reinterpret_cast<T*>(a.P);
   T* Q = reinterpret_cast<T*>(a.Q);
   Step st = step_of(a);
-  int64_t shift = a.shift;
+  WfBlocks bl = a.blocks;
   long long* prof = a.prof;
   unsigned* visits = a.visits;
   unsigned long long* upd = a.upd;
   int* owners = a.owners;
   unsigned* viol = a.viol;
   void* args[] = {&slots, &dup, &sub_off, &seq, &rank, &tickets, &s, &c, &P, &Q, &st,
-                  &shift, &prof, &visits, &upd, &owners, &viol};
+                  &bl, &prof, &visits, &upd, &owners, &viol};
   return cudaLaunchCooperativeKernel(reinterpret_cast<void*>(kern), blocks, threads, args, smem,
                                      a.stream);
 }
