@@ -601,7 +601,7 @@ def run_e2e(args, R, kw, stream, C):
     out = {"value": R.N / dt, "unit": "updates/s", "ms_per_step": 1000 * dt, "steps": steps,
            "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": 8 * world,
            "what": "per step: mf_train_epoch in out-of-core mode (staged=1: the epoch's ratings "
-                   "copied from pinned host memory, packed to 10 B per rating when n < 2^16, "
+                   "copied from pinned host memory, packed to 9-10 B per rating, "
                    "overlapped with compute) + mf_rmse (D2H); host wall clock, max over ranks"}
     if world > 1:
         return out

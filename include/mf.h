@@ -113,8 +113,10 @@ typedef struct mf_params {
                              HBM; a device set is preprocessed resident, then moved) and
                              each stratum's blocks stream into one of two HBM buffers on a copy
                              stream while the previous stratum computes; P, Q stay resident.
-                             When n <= 65535 the host copy and the H2D stream carry 10-B
-                             records (u int32, v uint16, r fp32) expanded on the GPU.
+                             The host copy and the H2D stream carry packed records: (u, v) as
+                             one integer of bits(m) + bits(n-1) bits in 5 bytes (<= 40 bits) or
+                             6 (<= 48), plus r fp32 -- 9 or 10 B per rating, expanded on the GPU
+                             (12-B slots beyond 48 bits).
                              Same order and result as resident.  0 = ratings resident in HBM */
   int32_t wf_kernel;      /* wavefront kernel: 0 = auto = 1 = ring-staged (cp.async smem ring),
                              2 = register pipeline; both give the same result                   */
@@ -240,8 +242,9 @@ typedef struct mf_stats {
   int64_t bytes_per_update; /* algorithmic: 12 + 4*k*sizeof(storage) (north_star; Eq. 5)  */
   int32_t workers, lanes, grid, block;
   int64_t h2d_bytes;        /* staged mode: bytes copied host -> device for the epoch's ratings
-                               (10 per rating when n <= 65535: packed u, v16, r; else 12; +2
-                               with the wavefront's duplicate distances)                      */
+                               (9 or 10 per rating packed, see params.staged; 12 unpacked; +2
+                               with the wavefront's duplicate distances; + P's row segments
+                               when staged = 2)                                                 */
 } mf_stats;
 mf_status mf_get_stats(mf_ctx* ctx, mf_stats* out);
 

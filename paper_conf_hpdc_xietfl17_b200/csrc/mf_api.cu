@@ -220,26 +220,45 @@ __global__ void k_dupdist(const Rating* __restrict__ slots, int64_t N, Grid G, i
   }
 }
 
-// Packed staging: 12-B slots <-> (u int32, v uint16, r fp32).  Sentinel pad slots (u = v = -1)
-// keep u = -1 and get v back from it; real v < n <= 65535.
-__global__ void k_split_slots(const Rating* __restrict__ s, int64_t N, int32_t* __restrict__ u,
-                              uint16_t* __restrict__ v, float* __restrict__ r) {
+// Packed staging records (the out-of-core H2D stream, section 6.2): (u, v) as ONE integer
+// uv = u << bv | v of bu + bv bits (bu = bits(m), bv = bits(n - 1)) stored in 4 + hib bytes --
+// a u32 low word and hib (1 or 2) high bytes -- plus r as fp32: 9 B per rating when
+// bu + bv <= 40 (Netflix, Yahoo shapes), 10 B up to 48 (Hugewiki), instead of the 12-B slot.
+// The sentinel pad slot (u = v = -1) is the all-ones uv: its u field 2^bu - 1 >= m is never a
+// real row.
+struct PackFmt {
+  int bu, bv, hib;
+};
+__global__ void k_split_slots(const Rating* __restrict__ s, int64_t N, PackFmt F,
+                              uint32_t* __restrict__ lo, uint8_t* __restrict__ hi,
+                              float* __restrict__ r) {
+  const uint64_t ones = (1ull << (F.bu + F.bv)) - 1ull;
   for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < N;
        x += (int64_t)gridDim.x * blockDim.x) {
     const Rating a = s[x];
-    u[x] = a.u;
-    v[x] = (uint16_t)a.v;
+    const uint64_t uv = a.u < 0 ? ones : (((uint64_t)(uint32_t)a.u << F.bv) | (uint32_t)a.v);
+    lo[x] = (uint32_t)uv;
+    if (F.hib == 1) {
+      hi[x] = (uint8_t)(uv >> 32);
+    } else {
+      reinterpret_cast<uint16_t*>(hi)[x] = (uint16_t)(uv >> 32);
+    }
     r[x] = a.r;
   }
 }
-__global__ void k_expand_slots(const int32_t* __restrict__ u, const uint16_t* __restrict__ v,
-                               const float* __restrict__ r, int64_t N, Rating* __restrict__ s) {
+__global__ void k_expand_slots(const uint32_t* __restrict__ lo, const uint8_t* __restrict__ hi,
+                               const float* __restrict__ r, int64_t N, PackFmt F,
+                               Rating* __restrict__ s) {
+  const uint32_t usent = (1u << F.bu) - 1u, vmask = (1u << F.bv) - 1u;
   for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < N;
        x += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t uu = __ldcs(u + x);
+    const uint64_t h = F.hib == 1 ? (uint64_t)__ldcs(hi + x)
+                                  : (uint64_t)__ldcs(reinterpret_cast<const unsigned short*>(hi) + x);
+    const uint64_t uv = (uint64_t)__ldcs(lo + x) | (h << 32);
+    const uint32_t u = (uint32_t)(uv >> F.bv);
     Rating a;
-    a.u = uu;
-    a.v = uu < 0 ? -1 : (int32_t)__ldcs(v + x);
+    a.u = u == usent ? -1 : (int32_t)u;
+    a.v = u == usent ? -1 : (int32_t)((uint32_t)uv & vmask);
     a.r = __ldcs(r + x);
     s[x] = a;
   }
@@ -671,11 +690,12 @@ struct mf_ctx {
   // (u int32, v uint16, r fp32, structure of arrays) instead of the 12-B slot; the compute
   // stream expands each staged stratum back into 12-B slots before its SGD launch.
   bool stg_packed = false;
-  int32_t* h_u = nullptr;
-  uint16_t* h_v16 = nullptr;
+  PackFmt pk{0, 0, 0};               // packed record format (bits of u, v; high bytes)
+  uint32_t* h_u = nullptr;           // packed: low words of uv
+  uint8_t* h_v16 = nullptr;          // packed: pk.hib high bytes of uv per rating
   float* h_r = nullptr;
-  int32_t* stg_u[2] = {nullptr, nullptr};
-  uint16_t* stg_v16[2] = {nullptr, nullptr};
+  uint32_t* stg_u[2] = {nullptr, nullptr};
+  uint8_t* stg_v16[2] = {nullptr, nullptr};
   float* stg_r[2] = {nullptr, nullptr};
   int64_t stg_len[2] = {0, 0};
   Rating* h_slots = nullptr;
@@ -1240,28 +1260,39 @@ static mf_status alloc_schedule(mf_ctx* c) {
   return MF_OK;
 }
 
+// The packed staging format of this ctx (k_split_slots): bu = bits(m), bv = bits(n - 1).
+static void set_pack_format(mf_ctx* c) {
+  const int bu = bits_for((uint64_t)c->m), bv = bits_for((uint64_t)std::max<int64_t>(c->n - 1, 1));
+  c->pk = PackFmt{bu, bv, bu + bv <= 40 ? 1 : 2};
+  c->stg_packed = bu + bv <= 48;
+}
+static int64_t staged_bytes_per_rating(const mf_ctx* c) {
+  return (c->stg_packed ? 8 + c->pk.hib : (int64_t)sizeof(Rating)) + (c->h_dup ? 2 : 0);
+}
+
 // Move the bucketed ratings (and the wavefront dup metadata) from HBM to pinned host memory
 // (the resident preprocessing path; the chunked path writes them there directly).
 static mf_status setup_staging(mf_ctx* c) {
   CUDA_TRY(c, cudaStreamSynchronize(c->st));
   const size_t ns = (size_t)std::max<int64_t>(c->nslots, 1);
-  c->stg_packed = c->n <= 65535;
+  set_pack_format(c);
   if (c->stg_packed) {
-    int32_t* du = nullptr;
-    uint16_t* dv = nullptr;
+    uint32_t* du = nullptr;
+    uint8_t* dv = nullptr;
     float* dr = nullptr;
+    const size_t hb = (size_t)c->pk.hib;
     TRY(c->alloc(&du, ns));
-    TRY(c->alloc(&dv, ns));
+    TRY(c->alloc(&dv, ns * hb));
     TRY(c->alloc(&dr, ns));
     if (c->nslots > 0) {
-      k_split_slots<<<grid_for(c->nslots, c->num_sms), 256, 0, c->st>>>(c->slots, c->nslots, du, dv, dr);
+      k_split_slots<<<grid_for(c->nslots, c->num_sms), 256, 0, c->st>>>(c->slots, c->nslots, c->pk, du, dv, dr);
       KERNEL_TRY(c);
     }
     CUDA_TRY(c, cudaMallocHost(&c->h_u, ns * 4));
-    CUDA_TRY(c, cudaMallocHost(&c->h_v16, ns * 2));
+    CUDA_TRY(c, cudaMallocHost(&c->h_v16, ns * hb));
     CUDA_TRY(c, cudaMallocHost(&c->h_r, ns * 4));
     CUDA_TRY(c, cudaMemcpyAsync(c->h_u, du, ns * 4, cudaMemcpyDeviceToHost, c->st));
-    CUDA_TRY(c, cudaMemcpyAsync(c->h_v16, dv, ns * 2, cudaMemcpyDeviceToHost, c->st));
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_v16, dv, ns * hb, cudaMemcpyDeviceToHost, c->st));
     CUDA_TRY(c, cudaMemcpyAsync(c->h_r, dr, ns * 4, cudaMemcpyDeviceToHost, c->st));
     CUDA_TRY(c, cudaStreamSynchronize(c->st));
     c->release(du);
@@ -1314,7 +1345,7 @@ static mf_status setup_staging_buffers(mf_ctx* c) {
     if (c->h_dup) TRY(c->alloc(&c->stg_dup[i], (size_t)cap));
     if (c->stg_packed) {
       TRY(c->alloc(&c->stg_u[i], (size_t)cap));
-      TRY(c->alloc(&c->stg_v16[i], (size_t)cap));
+      TRY(c->alloc(&c->stg_v16[i], (size_t)cap * c->pk.hib));
       TRY(c->alloc(&c->stg_r[i], (size_t)cap));
     }
     CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_h2d[i], cudaEventDisableTiming));
@@ -1347,8 +1378,8 @@ static mf_status stage(mf_ctx* c, int32_t t, int32_t j, int buf) {
     if (c->stg_packed) {
       CUDA_TRY(c, cudaMemcpyAsync(c->stg_u[buf] + off, c->h_u + lo, (size_t)len * 4,
                                   cudaMemcpyHostToDevice, c->cs));
-      CUDA_TRY(c, cudaMemcpyAsync(c->stg_v16[buf] + off, c->h_v16 + lo, (size_t)len * 2,
-                                  cudaMemcpyHostToDevice, c->cs));
+      CUDA_TRY(c, cudaMemcpyAsync(c->stg_v16[buf] + off * c->pk.hib, c->h_v16 + lo * c->pk.hib,
+                                  (size_t)len * c->pk.hib, cudaMemcpyHostToDevice, c->cs));
       CUDA_TRY(c, cudaMemcpyAsync(c->stg_r[buf] + off, c->h_r + lo, (size_t)len * 4,
                                   cudaMemcpyHostToDevice, c->cs));
     } else {
@@ -1358,7 +1389,7 @@ static mf_status stage(mf_ctx* c, int32_t t, int32_t j, int buf) {
     if (c->h_dup)
       CUDA_TRY(c, cudaMemcpyAsync(c->stg_dup[buf] + off, c->h_dup + lo, (size_t)len * 2,
                                   cudaMemcpyHostToDevice, c->cs));
-    c->h2d_bytes += len * (int64_t)((c->stg_packed ? 10 : sizeof(Rating)) + (c->h_dup ? 2 : 0));
+    c->h2d_bytes += len * staged_bytes_per_rating(c);
     off += len;
   }
   c->stg_len[buf] = off;
@@ -1406,7 +1437,8 @@ static mf_status stage_block(mf_ctx* c, int64_t b, int buf) {
   if (len == 0) return MF_OK;
   if (c->stg_packed) {
     CUDA_TRY(c, cudaMemcpyAsync(c->stg_u[buf], c->h_u + lo, (size_t)len * 4, cudaMemcpyHostToDevice, c->cs));
-    CUDA_TRY(c, cudaMemcpyAsync(c->stg_v16[buf], c->h_v16 + lo, (size_t)len * 2, cudaMemcpyHostToDevice, c->cs));
+    CUDA_TRY(c, cudaMemcpyAsync(c->stg_v16[buf], c->h_v16 + lo * c->pk.hib, (size_t)len * c->pk.hib,
+                                cudaMemcpyHostToDevice, c->cs));
     CUDA_TRY(c, cudaMemcpyAsync(c->stg_r[buf], c->h_r + lo, (size_t)len * 4, cudaMemcpyHostToDevice, c->cs));
   } else {
     CUDA_TRY(c, cudaMemcpyAsync(c->stg[buf], c->h_slots + lo, (size_t)len * sizeof(Rating),
@@ -1414,7 +1446,7 @@ static mf_status stage_block(mf_ctx* c, int64_t b, int buf) {
   }
   if (c->h_dup)
     CUDA_TRY(c, cudaMemcpyAsync(c->stg_dup[buf], c->h_dup + lo, (size_t)len * 2, cudaMemcpyHostToDevice, c->cs));
-  c->h2d_bytes += len * (int64_t)((c->stg_packed ? 10 : sizeof(Rating)) + (c->h_dup ? 2 : 0));
+  c->h2d_bytes += len * staged_bytes_per_rating(c);
   return MF_OK;
 }
 
@@ -1752,10 +1784,10 @@ static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, cons
   c->N = Nown;
   c->nslots = c->blk_off.back();
   const size_t ns = (size_t)std::max<int64_t>(c->nslots, 1);
-  c->stg_packed = c->n <= 65535;
+  set_pack_format(c);
   if (c->stg_packed) {
     CUDA_TRY(c, cudaMallocHost(&c->h_u, ns * 4));
-    CUDA_TRY(c, cudaMallocHost(&c->h_v16, ns * 2));
+    CUDA_TRY(c, cudaMallocHost(&c->h_v16, ns * (size_t)c->pk.hib));
     CUDA_TRY(c, cudaMallocHost(&c->h_r, ns * 4));
   } else {
     CUDA_TRY(c, cudaMallocHost(&c->h_slots, ns * sizeof(Rating)));
@@ -1772,8 +1804,8 @@ static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, cons
     Rating *r0 = nullptr, *r1 = nullptr;
     unsigned* cnt = nullptr;
     uint16_t* dd = nullptr;
-    int32_t* du = nullptr;
-    uint16_t* dv = nullptr;
+    uint32_t* du = nullptr;
+    uint8_t* dv = nullptr;
     float* dr = nullptr;
     TRY(c->alloc(&k0, (size_t)maxlen)); TRY(c->alloc(&k1, (size_t)maxlen));
     TRY(c->alloc(&i0, (size_t)maxlen)); TRY(c->alloc(&i1, (size_t)maxlen));
@@ -1784,7 +1816,7 @@ static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, cons
     }
     if (want_dup) TRY(c->alloc(&dd, (size_t)maxlen));
     if (c->stg_packed) {
-      TRY(c->alloc(&du, (size_t)maxlen)); TRY(c->alloc(&dv, (size_t)maxlen));
+      TRY(c->alloc(&du, (size_t)maxlen)); TRY(c->alloc(&dv, (size_t)maxlen * c->pk.hib));
       TRY(c->alloc(&dr, (size_t)maxlen));
     }
     std::vector<int64_t> subo;
@@ -1831,10 +1863,11 @@ static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, cons
         TRY(group_batches(c, fin, nullptr, padded));
       }
       if (c->stg_packed) {
-        k_split_slots<<<grid_for(padded, c->num_sms), 256, 0, c->st>>>(fin, padded, du, dv, dr);
+        k_split_slots<<<grid_for(padded, c->num_sms), 256, 0, c->st>>>(fin, padded, c->pk, du, dv, dr);
         KERNEL_TRY(c);
         CUDA_TRY(c, cudaMemcpyAsync(c->h_u + lo, du, (size_t)padded * 4, cudaMemcpyDeviceToHost, c->st));
-        CUDA_TRY(c, cudaMemcpyAsync(c->h_v16 + lo, dv, (size_t)padded * 2, cudaMemcpyDeviceToHost, c->st));
+        CUDA_TRY(c, cudaMemcpyAsync(c->h_v16 + lo * c->pk.hib, dv, (size_t)padded * c->pk.hib,
+                                    cudaMemcpyDeviceToHost, c->st));
         CUDA_TRY(c, cudaMemcpyAsync(c->h_r + lo, dr, (size_t)padded * 4, cudaMemcpyDeviceToHost, c->st));
       } else {
         CUDA_TRY(c, cudaMemcpyAsync(c->h_slots + lo, fin, (size_t)padded * sizeof(Rating),
@@ -2380,7 +2413,7 @@ static mf_status train_epoch_strata(mf_ctx* c, int32_t t, float g) {
       if (c->stg_packed) {
         if (c->stg_len[buf] > 0) {
           k_expand_slots<<<grid_for(c->stg_len[buf], c->num_sms), 256, 0, c->st>>>(
-              c->stg_u[buf], c->stg_v16[buf], c->stg_r[buf], c->stg_len[buf], c->stg[buf]);
+              c->stg_u[buf], c->stg_v16[buf], c->stg_r[buf], c->stg_len[buf], c->pk, c->stg[buf]);
           KERNEL_TRY(c);
           ++c->n_launch;
         }
@@ -2433,7 +2466,7 @@ static mf_status train_epoch_pq(mf_ctx* c, int32_t t, float g) {
       CUDA_TRY(c, cudaStreamWaitEvent(c->st, c->ev_pin[s], 0));
       if (c->stg_packed && c->stg_len[s] > 0) {
         k_expand_slots<<<grid_for(c->stg_len[s], c->num_sms), 256, 0, c->st>>>(
-            c->stg_u[s], c->stg_v16[s], c->stg_r[s], c->stg_len[s], c->stg[s]);
+            c->stg_u[s], c->stg_v16[s], c->stg_r[s], c->stg_len[s], c->pk, c->stg[s]);
         KERNEL_TRY(c);
         ++c->n_launch;
       }

@@ -749,8 +749,9 @@ def test_failed_load_releases_its_buffers_and_the_ctx_stays_usable():
 def test_staged_equals_resident(kw):
     """Section 6.2 out-of-core mode: ratings in pinned host memory, streamed per stratum through
     two HBM buffers (copy stream overlapping compute, also across epochs).  Same order, so the
-    deterministic result is bit-identical to the resident run.  n <= 65535 stages packed 10-B
-    records (expanded on the GPU); `wide` (n = 70,000) stages the 12-B slots as they are."""
+    deterministic result is bit-identical to the resident run.  The staged records are packed
+    to 9 B ((u, v) as one 17- or 26-bit integer in 5 bytes, r fp32; expanded on the GPU), also
+    for `wide` (n = 70,000)."""
     kw = dict(kw)
     k = kw.pop("k", 32)
     R = ragged() if not kw.pop("wide", False) else synth.uniform(
@@ -763,8 +764,8 @@ def test_staged_equals_resident(kw):
         for _ in range(3):
             g.train_epoch()
         if staged:
-            per = 10 if R.n <= 65535 else 12
-            per += 2 if kw["schedule"] == "wavefront" else 0
+            # packed records: uv in bits(m) + bits(n - 1) <= 40 bits -> 5 bytes, + fp32 r
+            per = 9 + (2 if kw["schedule"] == "wavefront" else 0)
             h2d = g.stats()["h2d_bytes"]      # ~ one epoch: its later strata + the next epoch's first
             assert h2d % per == 0 and 0.5 * R.N <= h2d / per <= 1.5 * R.N, (h2d, per)
         out.append((g.factors(), g.rmse()))
