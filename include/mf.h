@@ -145,7 +145,10 @@ typedef struct mf_params {
                              streaming loads + warp shuffles; 1 = TMA: one lane per worker
                              bulk-copies its chunk into shared memory in 768-B sub-chunks
                              (cp.async.bulk + mbarrier, double buffered).  1 needs f % 64 == 0,
-                             prefetch 1 and the default 16-B lanes (else MF_E_UNSUPPORTED)    */
+                             prefetch 1 and the default 16-B lanes (else MF_E_UNSUPPORTED).
+                             2 = the next 2 samples' p/q rows copied into a per-worker shared-
+                             memory ring by cp.async (a deeper row pipeline without registers;
+                             16-B lane slices, k S >= 256).  All three: same order and result */
   int64_t stage_chunk;    /* staged = 1 with a HOST train set: samples per chunk of the
                              out-of-core preprocessing (0 = 2^26).  Device memory then holds one
                              chunk (~68 B per sample) or one strata block (~60 B per sample) at a

@@ -966,7 +966,8 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->check_owners < 0 || p->check_owners > 1) return MF_E_INVAL;
   if (p->group_cols && (p->schedule != MF_HOGWILD || p->rating_stage || p->prefetch > 1))
     return MF_E_UNSUPPORTED;
-  if (p->rating_stage < 0 || p->rating_stage > 1) return MF_E_INVAL;
+  if (p->rating_stage < 0 || p->rating_stage > 2) return MF_E_INVAL;
+  if (p->rating_stage == 2 && (p->lane_bytes && p->lane_bytes != 16)) return MF_E_UNSUPPORTED;
   if (p->rating_stage == 1 && ((p->batch_f > 0 ? p->batch_f : 256) % 64 != 0 ||
                                p->prefetch > 1 || (p->lane_bytes && p->lane_bytes != 16)))
     return MF_E_UNSUPPORTED;                      // TMA stream: f % 64 == 0, default geometry

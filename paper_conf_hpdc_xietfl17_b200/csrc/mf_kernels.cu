@@ -57,6 +57,11 @@ __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L >
   extern __shared__ __align__(16) char hsm[];
   RatingRing ring{};
   unsigned phase = 0;
+  char* rowring = nullptr;                           // SRC = 2: this group's row ring (2F slots)
+  if constexpr (SRC == 2) {
+    const int gid = (int)(threadIdx.x >> 5) * GPW + grp;
+    rowring = hsm + (size_t)gid * 4 * 2 * K * sizeof(T);
+  }
   if constexpr (SRC == 1) {
     const int gid = (int)(threadIdx.x >> 5) * GPW + grp;   // group within the CTA
     const int ngroups = (int)(blockDim.x >> 5) * GPW;
@@ -88,8 +93,11 @@ __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L >
       if (gl == 0) atomicAdd(visits + chunk, 1u);    // exactly-once evidence (mf_check_visits)
     }
     // every group of the warp runs f iterations in lockstep (inactive ones on sentinels)
-    done += run_serial<T, K, L, D, true, ADA, EX, SRC, GRP>(slots, lo, f, act, P, Q, st, gl, gbase,
-                                                       0xffffffffu, ada, ring, &phase);
+    if constexpr (SRC == 2)
+      done += run_chunk_ring<T, K, L, 2, EX>(slots, lo, f, act, P, Q, st, gl, gbase, rowring);
+    else
+      done += run_serial<T, K, L, D, true, ADA, EX, SRC, GRP>(slots, lo, f, act, P, Q, st, gl, gbase,
+                                                         0xffffffffu, ada, ring, &phase);
   }
   if (gl == 0 && done) atomicAdd(upd, (unsigned long long)done);
 }
@@ -519,10 +527,12 @@ static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
   auto kern = k_hogwild<T, K, L, D, ADA, EX, SRC, GRP>;
   const int threads = 256;
   const int groups = threads / 32 * (32 / L);
-  const size_t smem = SRC == 1 ? (size_t)groups * (16 + 2 * kSubBytes) : 0;
+  const size_t smem = SRC == 1   ? (size_t)groups * (16 + 2 * kSubBytes)
+                      : SRC == 2 ? (size_t)groups * 4 * 2 * K * sizeof(T)
+                                 : 0;
   cudaError_t e;
-  if (SRC == 1) {
-    if (a.f % kSub != 0) return cudaErrorInvalidValue;     // mf_create rejects it first
+  if (SRC != 0) {
+    if (SRC == 1 && a.f % kSub != 0) return cudaErrorInvalidValue;   // mf_create rejects it first
     e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     // the rings need the shared-memory carveout that keeps MF_HOG_MINB blocks resident
@@ -667,6 +677,8 @@ static cudaError_t hogwild_kl(const HogwildLaunch& a) {
   if (a.exact) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, true>(a);  // depth 1
   if (a.rating_stage == 1 && LB == 16)
     return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, false, 1>(a);        // TMA stream
+  if constexpr ((K * S) / lanes_for(K, S, LB) == 16)
+    if (a.rating_stage == 2) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, false, 2>(a);
   if (a.prefetch == 1) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1>(a);
   return launch_hogwild_t<T, K, lanes_for(K, S, LB), 2>(a);
 }

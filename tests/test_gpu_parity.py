@@ -315,17 +315,22 @@ def test_appendix_a_hand_pins_through_the_abi(golden_dir):
                                 dict(k=32, storage="fp16"), dict(k=256, storage="bf16"),
                                 dict(k=64, storage="fp32", grid_a=4, batch_f=128),
                                 dict(k=128, storage="fp16", grid_a=4, batch_f=64, staged=True)])
-def test_tma_rating_stream_equals_register_stream(kw):
+@pytest.mark.parametrize("stage", [1, 2])
+def test_tma_rating_stream_equals_register_stream(kw, stage):
     """rating_stage = 1 (the chunk's ratings bulk-copied into shared memory by the TMA engine,
-    768-B sub-chunks, mbarrier-tracked, double buffered) feeds the same samples in the same
-    order as the per-lane load + shuffle stream: 1-worker runs are bit-identical, and both
-    match the oracle (fp32: 1e-4); at full concurrency every chunk is claimed once."""
+    768-B sub-chunks, mbarrier-tracked, double buffered) and rating_stage = 2 (the next 2
+    samples' rows copied into a per-worker shared-memory ring by cp.async) feed the same samples
+    in the same order with the same arithmetic as the register kernel: 1-worker runs are
+    bit-identical, and both match the oracle (fp32: 1e-4); at full concurrency every chunk is
+    claimed once."""
     kw = dict(kw)
     k = kw.pop("k")
+    if stage == 2 and k * (2 if kw["storage"] != "fp32" else 4) < 256:
+        pytest.skip("the row ring needs 16-B lane slices (k S >= 256)")
     R = ragged()
     out = []
-    for stage in (0, 1):
-        g = mf.MF(R.m, R.n, k, workers=1, rating_stage=stage, **TABLE3_NETFLIX, **kw)
+    for st_ in (0, stage):
+        g = mf.MF(R.m, R.n, k, workers=1, rating_stage=st_, **TABLE3_NETFLIX, **kw)
         g.load(R.u, R.v, R.r)
         g.load(R.ut, R.vt, R.rt, "test")
         for _ in range(2):
@@ -343,7 +348,7 @@ def test_tma_rating_stream_equals_register_stream(kw):
         o.train_epoch()
         Po, Qo = o.factors()
         assert np.abs(P1 - Po).max() <= 1e-4 and np.abs(Q1 - Qo).max() <= 1e-4
-    g = mf.MF(R.m, R.n, k, rating_stage=1, **TABLE3_NETFLIX, **kw)    # all resident workers
+    g = mf.MF(R.m, R.n, k, rating_stage=stage, **TABLE3_NETFLIX, **kw)   # all resident workers
     g.load(R.u, R.v, R.r)
     for _ in range(3):
         g.train_epoch()
