@@ -29,7 +29,8 @@ def pair(R, k=16, **kw):
     if R.ut is not None:
         g.load(R.ut, R.vt, R.rt, "test")
     okw = {kk: vv for kk, vv in kw.items() if kk not in ("lane_bytes", "prefetch", "wf_kernel", "staged", "exact_order",
-                                                          "launch_blocks")}
+                                                          "launch_blocks", "rating_stage", "stage_chunk",
+                                                          "check_owners")}
     if kw.get("schedule") == "wavefront":
         okw.setdefault("workers", kw.get("workers"))
     o = po.Oracle(R.m, R.n, k, R.u, R.v, R.r, **okw)
@@ -693,6 +694,33 @@ def test_p_out_of_core_below_the_device_budget_is_bit_identical(kw):
     assert np.array_equal(P0, P1) and np.array_equal(Q0, Q1)
     # the segment-by-segment RMSE sums the same squared errors in another order
     assert abs(i0 - i1) <= 1e-12 * i0 and abs(r0 - r1) <= 1e-12 * r0, (i0, i1, r0, r1)
+
+
+@pytest.mark.parametrize("N", [1, 5, 300, 1000])
+@pytest.mark.parametrize("kw", [dict(schedule="hogwild", staged=1, stage_chunk=1, grid_a=2, batch_f=64),
+                                dict(schedule="hogwild", staged=2, stage_chunk=7, grid_a=4, batch_f=32),
+                                dict(schedule="wavefront", staged=2, stage_chunk=3, grid_a=2, workers=3,
+                                     wf_cols=4),
+                                dict(schedule="hogwild", group_cols=True, batch_f=64, grid_a=2),
+                                dict(schedule="hogwild", rating_stage=2, k=128, storage="fp16"),
+                                dict(schedule="hogwild", rating_stage=1, batch_f=64, k=128, storage="fp16")])
+def test_edge_sizes_of_the_round2_paths(N, kw):
+    """Tiny and ragged sets (N = 1, N < f, empty strata blocks, chunks of 1 sample) through the
+    chunked loader, P out of core, grouped batches and both staged rating streams: the 1-worker
+    result equals the oracle (fp32 1e-5 / low precision 2 ulps) and every unit is claimed once."""
+    kw = dict(kw)
+    k = kw.pop("k", 16)
+    R = synth.uniform(m=40, n=30, N=N, seed=N + 1, mu=0.3, rank=2, noise=0.1, Ntest=50)
+    g, o = pair(R, k=k, workers=kw.pop("workers", 1), **TABLE3_NETFLIX, **kw)
+    for _ in range(2):
+        g.train_epoch()
+        o.train_epoch()
+        assert g.stats()["updates"] == N
+    assert g.check_visits()["bad_units"] == 0
+    tol = 1e-5 if kw.get("storage", "fp32") == "fp32" else 2e-3
+    for Xg, Xo in zip(g.factors(), o.factors()):
+        assert np.abs(Xg - Xo).max() <= tol
+    assert abs(g.rmse() - o.rmse(R.ut, R.vt, R.rt)) <= 1e-4 * o.rmse(R.ut, R.vt, R.rt)
 
 
 def test_resident_load_fails_cleanly_below_the_device_budget():
