@@ -358,6 +358,10 @@ def ncu_traffic(args):
         d = json.load(f)
     key = f"{args.workload}/{args.schedule}/{args.storage}/k{args.k}"
     e = d.get(key, {})
+    # a capture describes one launch configuration: plain or grouped batches of f, full size
+    if (e.get("batch_f", 256) != default_f(args, 1) or e.get("group_cols", False) != bool(args.group_cols)
+            or e.get("fraction", 1.0) != args.fraction):
+        return None, None
     return e.get("dram_bytes_per_launch"), e.get("source")
 
 
