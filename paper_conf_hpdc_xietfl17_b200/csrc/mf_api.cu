@@ -1056,6 +1056,25 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   return MF_OK;
 }
 
+// The out-of-core state a train load creates outside the allocator: pinned host copies of the
+// ratings and P, the copy / write-back streams and their events.  Streams must be idle.
+static void release_host_staging(mf_ctx* c) {
+  for (void** h : {(void**)&c->h_slots, (void**)&c->h_u, (void**)&c->h_v16, (void**)&c->h_r,
+                   (void**)&c->h_dup, (void**)&c->h_P}) {
+    if (*h) cudaFreeHost(*h);
+    *h = nullptr;
+  }
+  for (int i = 0; i < 2; ++i)
+    for (cudaEvent_t* e : {&c->ev_pin[i], &c->ev_pcomp[i], &c->ev_pout[i], &c->ev_h2d[i], &c->ev_free[i]}) {
+      if (*e) cudaEventDestroy(*e);
+      *e = nullptr;
+    }
+  for (cudaStream_t* q : {&c->ds, &c->cs}) {
+    if (*q) cudaStreamDestroy(*q);
+    *q = nullptr;
+  }
+}
+
 void mf_destroy(mf_ctx* c) {
   if (!c) return;
   cudaSetDevice(c->dev);
@@ -1076,21 +1095,7 @@ void mf_destroy(mf_ctx* c) {
   for (cudaEvent_t e : {c->ev_e0, c->ev_e1, c->ev_s0, c->ev_s1, c->ev_c0, c->ev_c1})
     if (e) cudaEventDestroy(e);
   if (c->comm) mf::Comm::destroy(c->comm);
-  if (c->h_slots) cudaFreeHost(c->h_slots);
-  if (c->h_u) cudaFreeHost(c->h_u);
-  if (c->h_v16) cudaFreeHost(c->h_v16);
-  if (c->h_r) cudaFreeHost(c->h_r);
-  if (c->h_dup) cudaFreeHost(c->h_dup);
-  if (c->h_P) cudaFreeHost(c->h_P);
-  for (int i = 0; i < 2; ++i)
-    for (cudaEvent_t e : {c->ev_pin[i], c->ev_pcomp[i], c->ev_pout[i]})
-      if (e) cudaEventDestroy(e);
-  if (c->ds) cudaStreamDestroy(c->ds);
-  for (int i = 0; i < 2; ++i) {
-    if (c->ev_h2d[i]) cudaEventDestroy(c->ev_h2d[i]);
-    if (c->ev_free[i]) cudaEventDestroy(c->ev_free[i]);
-  }
-  if (c->cs) cudaStreamDestroy(c->cs);
+  release_host_staging(c);
   for (cudaEvent_t e : {c->ev_ss_go, c->ev_ss_done})
     if (e) cudaEventDestroy(e);
   if (c->ss) cudaStreamDestroy(c->ss);
@@ -2019,7 +2024,10 @@ mf_status mf_load_coo(mf_ctx* c, int32_t set, int64_t nnz, const int32_t* u, con
   if (s != MF_OK && c->sticky == MF_OK) {
     // recoverable failure (MF_E_RANGE, MF_E_NOMEM, ...): the ctx stays usable
     cudaStreamSynchronize(c->st);
+    if (c->cs) cudaStreamSynchronize(c->cs);
+    if (c->ds) cudaStreamSynchronize(c->ds);
     c->drop_allocations_since(before);
+    if (set == MF_TRAIN) release_host_staging(c);   // a retried load allocates them again
   }
   return s;
 }

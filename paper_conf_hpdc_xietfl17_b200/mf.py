@@ -156,12 +156,13 @@ class _TorchAllocator:
     def __init__(self, device: int, budget: int | None = None):
         torch = _torch()
         self.device = device
+        self.budget = budget              # may be raised between a failed and a retried load
         self.sizes = {}
         self.live = 0
         self.peak = 0
 
         def _alloc(nbytes, stream, user):
-            if budget is not None and self.live + int(nbytes) > budget:
+            if self.budget is not None and self.live + int(nbytes) > self.budget:
                 return None
             try:
                 ptr = torch.cuda.caching_allocator_alloc(int(nbytes), device, int(stream or 0))

@@ -723,6 +723,33 @@ def test_edge_sizes_of_the_round2_paths(N, kw):
     assert abs(g.rmse() - o.rmse(R.ut, R.vt, R.rt)) <= 1e-4 * o.rmse(R.ut, R.vt, R.rt)
 
 
+@pytest.mark.parametrize("staged", [1, 2])
+def test_out_of_core_load_retried_after_nomem_matches_a_fresh_ctx(staged):
+    """A chunked out-of-core load that runs out of device budget part-way (MF_E_NOMEM) releases
+    what it took -- device buffers, pinned host copies, copy streams -- and the same ctx, given
+    more budget, loads again and trains bit-identically to a fresh ctx."""
+    R = synth.uniform(m=3000, n=900, N=400_000, seed=5, mu=0.5, rank=4, noise=0.1, Ntest=2000)
+    kw = dict(grid_a=4, batch_f=64, staged=staged, stage_chunk=1 << 16, workers=1, seed=9)
+    ok = mf.MF(R.m, R.n, 32, **TABLE3_NETFLIX, **kw)
+    ok.load(R.u, R.v, R.r)
+    need = ok.device_peak_bytes
+    ok.train_epoch()
+    want = ok.factors()
+    ok.close()
+    for budget in (need // 3, need * 9 // 10, need - 1):      # early and late failure points
+        g = mf.MF(R.m, R.n, 32, device_budget=budget, **TABLE3_NETFLIX, **kw)
+        with pytest.raises(mf.MFError) as e:
+            g.load(R.u, R.v, R.r)
+        assert e.value.status == -2
+        assert g._alloc.live < budget
+        g._alloc.budget = None
+        g.load(R.u, R.v, R.r)
+        g.train_epoch()
+        for Xg, Xw in zip(g.factors(), want):
+            assert np.array_equal(Xg, Xw)
+        g.close()
+
+
 def test_resident_load_fails_cleanly_below_the_device_budget():
     """The same budget without out-of-core staging: the resident preprocessing needs the whole
     set in HBM, so the load fails with MF_E_NOMEM (and the ctx stays usable)."""
