@@ -148,7 +148,10 @@ typedef struct mf_params {
                              prefetch 1 and the default 16-B lanes (else MF_E_UNSUPPORTED).
                              2 = the next 2 samples' p/q rows copied into a per-worker shared-
                              memory ring by cp.async (a deeper row pipeline without registers;
-                             16-B lane slices, k S >= 256).  All three: same order and result */
+                             16-B lane slices: k S <= 512, prefetch 1).  1 and 2 are Hogwild
+                             with the Eq. 9 step in the fast form only (exact_order, ADAGRAD or
+                             another schedule: MF_E_UNSUPPORTED).  All three: same order and
+                             result                                                          */
   int64_t stage_chunk;    /* staged = 1 with a HOST train set: samples per chunk of the
                              out-of-core preprocessing (0 = 2^26).  Device memory then holds one
                              chunk (~68 B per sample) or one strata block (~60 B per sample) at a

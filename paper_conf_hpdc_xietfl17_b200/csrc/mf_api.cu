@@ -967,7 +967,13 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->group_cols && (p->schedule != MF_HOGWILD || p->rating_stage || p->prefetch > 1))
     return MF_E_UNSUPPORTED;
   if (p->rating_stage < 0 || p->rating_stage > 2) return MF_E_INVAL;
-  if (p->rating_stage == 2 && (p->lane_bytes && p->lane_bytes != 16)) return MF_E_UNSUPPORTED;
+  // the staged rating streams are instantiated for plain Eq. 9 updates in the fast form only;
+  // the row ring (2) needs 16-B lane slices: k S <= 512 at the default 16-B lanes
+  if (p->rating_stage && (p->exact_order || p->lr_rule == 1 || p->schedule != MF_HOGWILD))
+    return MF_E_UNSUPPORTED;
+  if (p->rating_stage == 2 && ((p->lane_bytes && p->lane_bytes != 16) || p->prefetch > 1 ||
+                               (int64_t)p->k * (p->storage == MF_FP32 ? 4 : 2) > 512))
+    return MF_E_UNSUPPORTED;
   if (p->rating_stage == 1 && ((p->batch_f > 0 ? p->batch_f : 256) % 64 != 0 ||
                                p->prefetch > 1 || (p->lane_bytes && p->lane_bytes != 16)))
     return MF_E_UNSUPPORTED;                      // TMA stream: f % 64 == 0, default geometry

@@ -77,6 +77,27 @@ def test_create_rejects_bad_params_before_touching_a_device(L):
     assert not h.value
 
 
+def test_create_refuses_combinations_no_kernel_implements(L):
+    """Options that have no kernel instantiation are refused with MF_E_UNSUPPORTED at create
+    (never silently run as another variant)."""
+    def refused(**kw):
+        p = mf.Params()
+        L.mf_params_default(ctypes.byref(p))
+        p.m, p.n = 1000, 800
+        for kk, vv in kw.items():
+            setattr(p, kk, vv)
+        h = ctypes.c_void_p()
+        return L.mf_create(ctypes.byref(p), ctypes.byref(h)) == -7 and not h.value
+    assert refused(rating_stage=1, exact_order=1)
+    assert refused(rating_stage=2, lr_rule=1)
+    assert refused(rating_stage=1, schedule=1)                        # wavefront
+    assert refused(rating_stage=2, k=256, storage=0)                  # 32-B lane slices
+    assert refused(rating_stage=2, prefetch=2)
+    assert refused(rating_stage=1, batch_f=100)                       # f % 64 != 0
+    assert refused(group_cols=1, schedule=1)
+    assert refused(staged=2, world=2, grid_a=8, rank=0)
+
+
 def test_strata_holders_partition_and_rotation(L):
     """A: in sub-epoch j segment J is held by the owner of row (J - pi_t[j]) mod a; each rank
     holds exactly a/G segments per sub-epoch; pi_t is the oracle's strata order."""

@@ -326,8 +326,6 @@ def test_tma_rating_stream_equals_register_stream(kw, stage):
     claimed once."""
     kw = dict(kw)
     k = kw.pop("k")
-    if stage == 2 and k * (2 if kw["storage"] != "fp32" else 4) < 256:
-        pytest.skip("the row ring needs 16-B lane slices (k S >= 256)")
     R = ragged()
     out = []
     for st_ in (0, stage):
