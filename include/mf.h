@@ -293,6 +293,18 @@ mf_status mf_strata_plan(uint64_t seed, int32_t a, int32_t world, int32_t rank, 
                          int32_t t, int32_t j, int32_t* holders, int64_t* blocks,
                          int32_t* nblocks, int64_t* xfers, int32_t* nxfers);
 
+/* Debug / test surface: run every primitive of the strata mode's transport (a12; section 6.1,
+ * P:L305-316 adapted) outside a training context and check the results: the fp64 all-reduce
+ * of the RMSE, a broadcast, one grouped send/recv set shaped like a Q-segment rotation
+ * (segment r moves r -> (r+1) mod world), and the segment gather of mf_get_factors.  Each of
+ * the `world` ranks calls it on its own `device` with the same 128-byte ncclUniqueId (transport
+ * 0 = NCCL) or loopback group key (1, ranks = threads of one process).  world = 1 is valid and
+ * runs every NCCL call on one GPU (the rotation becomes a send/recv to self).  Synchronises.
+ * Returns MF_OK when every value checks, MF_E_NCCL / MF_E_CUDA on a failed call, MF_E_RANGE
+ * on a wrong value; `msg` (msg_len bytes, may be NULL) receives a one-line report. */
+mf_status mf_comm_selftest(const void* comm_id, int32_t world, int32_t rank, int32_t device,
+                           int32_t transport, char* msg, int32_t msg_len);
+
 void mf_destroy(mf_ctx* ctx);
 const char* mf_last_error(const mf_ctx* ctx);
 const char* mf_status_string(mf_status s);

@@ -938,6 +938,102 @@ mf_status mf_strata_plan(uint64_t seed, int32_t a, int32_t world, int32_t rank, 
   return MF_OK;
 }
 
+mf_status mf_comm_selftest(const void* comm_id, int32_t world, int32_t rank, int32_t device,
+                           int32_t transport, char* msg, int32_t msg_len) {
+  std::string text;
+  auto done = [&](mf_status s, const std::string& t) {
+    if (msg && msg_len > 0) std::snprintf(msg, (size_t)msg_len, "%s", t.c_str());
+    return s;
+  };
+  if (!comm_id || world < 1 || rank < 0 || rank >= world || transport < 0 || transport > 1)
+    return done(MF_E_INVAL, "bad arguments");
+  if (cudaSetDevice(device) != cudaSuccess) return done(MF_E_CUDA, "cudaSetDevice failed");
+  cudaStream_t st = nullptr;
+  if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess)
+    return done(MF_E_CUDA, "cudaStreamCreate failed");
+  uint8_t id[128];
+  std::memcpy(id, comm_id, 128);
+  std::string why;
+  mf::Comm* cm = transport == 1 ? mf::Comm::create_loopback(id, world, rank, st, &why)
+                                : mf::Comm::create(id, world, rank, st, &why);
+  if (!cm) {
+    cudaStreamDestroy(st);
+    return done(MF_E_NCCL, "communicator: " + why);
+  }
+  const size_t seg = 4096, rowb = 16;
+  const int64_t rows = 3 * (int64_t)world + 1;
+  auto pat = [](int r) { return (unsigned char)(r * 13 + 1); };
+  double* d = nullptr;
+  unsigned char *buf = nullptr, *bc = nullptr, *rw = nullptr;
+  mf_status s = MF_OK;
+  bool ok = cudaMalloc(&d, 4 * sizeof(double)) == cudaSuccess &&
+            cudaMalloc(&buf, seg * (size_t)world) == cudaSuccess &&
+            cudaMalloc(&bc, seg) == cudaSuccess &&
+            cudaMalloc(&rw, rowb * (size_t)rows) == cudaSuccess;
+  std::vector<double> hd(4);
+  for (int i = 0; i < 4; ++i) hd[(size_t)i] = (double)(rank + 1) * (i + 1);
+  ok = ok && cudaMemcpyAsync(d, hd.data(), 4 * sizeof(double), cudaMemcpyHostToDevice, st) == cudaSuccess;
+  ok = ok && cudaMemsetAsync(bc, pat(rank), seg, st) == cudaSuccess;
+  ok = ok && cudaMemsetAsync(buf, 0xEE, seg * (size_t)world, st) == cudaSuccess;
+  ok = ok && cudaMemsetAsync(buf + seg * (size_t)rank, pat(rank), seg, st) == cudaSuccess;
+  ok = ok && cudaMemsetAsync(rw, 0, rowb * (size_t)rows, st) == cudaSuccess;
+  const int64_t lo = cdiv64((int64_t)rank * rows, world), hi = cdiv64((int64_t)(rank + 1) * rows, world);
+  if (hi > lo) ok = ok && cudaMemsetAsync(rw + lo * rowb, pat(rank), (size_t)(hi - lo) * rowb, st) == cudaSuccess;
+  if (!ok) s = MF_E_CUDA, text = "device buffers";
+  std::vector<mf::Xfer> xs;
+  for (int r = 0; r < world; ++r) xs.push_back(mf::Xfer{buf + seg * (size_t)r, seg, r, (r + 1) % world});
+  if (s == MF_OK && !cm->allreduce_sum(d, 4, &why)) s = MF_E_NCCL, text = "all-reduce: " + why;
+  if (s == MF_OK && !cm->broadcast(bc, seg, world - 1, &why)) s = MF_E_NCCL, text = "broadcast: " + why;
+  if (s == MF_OK && !cm->exchange(xs, rank, &why)) s = MF_E_NCCL, text = "send/recv: " + why;
+  if (s == MF_OK && !cm->gather_rows(rw, rows, world, world, rowb, &why)) s = MF_E_NCCL, text = "gather: " + why;
+  std::vector<unsigned char> hb(seg * (size_t)world), hc(seg), hr(rowb * (size_t)rows);
+  if (s == MF_OK) {
+    ok = cudaMemcpyAsync(hd.data(), d, 4 * sizeof(double), cudaMemcpyDeviceToHost, st) == cudaSuccess &&
+         cudaMemcpyAsync(hb.data(), buf, hb.size(), cudaMemcpyDeviceToHost, st) == cudaSuccess &&
+         cudaMemcpyAsync(hc.data(), bc, seg, cudaMemcpyDeviceToHost, st) == cudaSuccess &&
+         cudaMemcpyAsync(hr.data(), rw, hr.size(), cudaMemcpyDeviceToHost, st) == cudaSuccess &&
+         cudaStreamSynchronize(st) == cudaSuccess;
+    if (!ok) s = MF_E_CUDA, text = "read-back";
+  }
+  if (s == MF_OK) {
+    const double tri = (double)world * (world + 1) / 2.0;
+    for (int i = 0; i < 4 && s == MF_OK; ++i)
+      if (hd[(size_t)i] != tri * (i + 1)) s = MF_E_RANGE, text = "all-reduce value";
+    for (size_t x = 0; x < seg && s == MF_OK; ++x)
+      if (hc[x] != pat(world - 1)) s = MF_E_RANGE, text = "broadcast value";
+    const int from = (rank + world - 1) % world;
+    for (int r = 0; r < world && s == MF_OK; ++r) {
+      const unsigned char want = (r == rank || r == from) ? pat(r) : 0xEE;
+      for (size_t x = 0; x < seg; ++x)
+        if (hb[seg * (size_t)r + x] != want) {
+          s = MF_E_RANGE, text = "send/recv value";
+          break;
+        }
+    }
+    for (int r = 0; r < world && s == MF_OK; ++r) {
+      const int64_t a0 = cdiv64((int64_t)r * rows, world), a1 = cdiv64((int64_t)(r + 1) * rows, world);
+      for (int64_t x = a0 * (int64_t)rowb; x < a1 * (int64_t)rowb; ++x)
+        if (hr[(size_t)x] != pat(r)) {
+          s = MF_E_RANGE, text = "gather value";
+          break;
+        }
+    }
+  }
+  if (s == MF_OK) {
+    char line[160];
+    std::snprintf(line, sizeof(line), "ok: %s, rank %d of %d: all-reduce, broadcast, %d-segment send/recv, "
+                  "%lld-row gather checked", transport ? "loopback" : "NCCL", rank, world, world,
+                  (long long)rows);
+    text = line;
+  }
+  mf::Comm::destroy(cm);
+  for (void* x : {(void*)d, (void*)buf, (void*)bc, (void*)rw})
+    if (x) cudaFree(x);
+  cudaStreamDestroy(st);
+  cudaGetLastError();
+  return done(s, text);
+}
+
 mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (!out) return MF_E_INVAL;
   *out = nullptr;

@@ -73,7 +73,7 @@ EXPORTED = ["mf_abi_version", "mf_params_default", "mf_create", "mf_load_coo", "
             "mf_rmse", "mf_loss", "mf_get_factors", "mf_set_factors", "mf_set_epoch", "mf_get_epoch",
             "mf_export_schedule", "mf_get_stats", "mf_get_launch_ms", "mf_check_visits",
             "mf_owner_violations",
-            "mf_strata_holders", "mf_strata_plan",
+            "mf_strata_holders", "mf_strata_plan", "mf_comm_selftest",
             "mf_destroy",
             "mf_last_error", "mf_status_string"]
 
@@ -107,6 +107,7 @@ def lib() -> ctypes.CDLL:
         "mf_owner_violations": (i32, [vp, ctypes.POINTER(i64)]),
         "mf_strata_holders": (i32, [u64, i32, i32, i32, i32, vp]),
         "mf_strata_plan": (i32, [u64, i32, i32, i32, i64, i32, i32, vp, vp, vp, vp, vp]),
+        "mf_comm_selftest": (i32, [vp, i32, i32, i32, i32, ctypes.c_char_p, i32]),
         "mf_destroy": (None, [vp]),
         "mf_last_error": (ctypes.c_char_p, [vp]),
         "mf_status_string": (ctypes.c_char_p, [i32]),
@@ -141,6 +142,20 @@ def strata_plan(seed: int, a: int, world: int, rank: int, n: int, t: int, j: int
         raise MFError(st, "mf_strata_plan")
     tr = [tuple(xf[5 * i:5 * i + 5]) for i in range(nx.value)]
     return list(blocks[:nb.value]), tr, list(h)
+
+
+def comm_selftest(comm_id: bytes, world: int = 1, rank: int = 0, device: int = 0,
+                  transport: int = 0) -> str:
+    """Run the strata transport's primitives (all-reduce, broadcast, rotation-shaped send/recv,
+    segment gather) on `device` and check them (mf_comm_selftest); returns the report line,
+    raises MFError on a failed call or a wrong value."""
+    idb = ctypes.create_string_buffer(bytes(comm_id).ljust(128, b"\0")[:128], 128)
+    out = ctypes.create_string_buffer(256)
+    st = lib().mf_comm_selftest(ctypes.cast(idb, ctypes.c_void_p), world, rank, device, transport,
+                                out, 256)
+    if st != 0:
+        raise MFError(st, "mf_comm_selftest: " + out.value.decode(errors="replace"))
+    return out.value.decode()
 
 
 def _torch():
@@ -458,6 +473,7 @@ def mf_destroy(ctx: MF) -> None:
 
 mf_strata_holders = strata_holders
 mf_strata_plan = strata_plan
+mf_comm_selftest = comm_selftest
 
 
 def _is_cuda_tensor(x) -> bool:

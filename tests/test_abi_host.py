@@ -115,3 +115,12 @@ def test_strata_holders_partition_and_rotation(L):
                     assert h[J] == r // (a // G)
     with pytest.raises(mf.MFError):
         mf.strata_holders(42, 8, 3, 0, 0)
+
+
+def test_comm_selftest_rejects_bad_arguments_before_touching_a_device(L):
+    buf = ctypes.create_string_buffer(128)
+    out = ctypes.create_string_buffer(64)
+    assert L.mf_comm_selftest(None, 1, 0, 0, 0, out, 64) == -1
+    assert L.mf_comm_selftest(buf, 2, 2, 0, 0, out, 64) == -1          # rank >= world
+    assert L.mf_comm_selftest(buf, 1, 0, 0, 3, out, 64) == -1          # transport
+    assert out.value == b"bad arguments"
