@@ -66,6 +66,9 @@ typedef struct or_params {
   float   ada_eps;         /* ADAGRAD epsilon */
   int32_t group_cols;      /* batch-Hogwild, reading R24: inside each batch of f consecutive
                               samples, update them in order of (relabelled column, position) */
+  int32_t grid_cols;       /* column segments of the grid: 0 = a (the a x a strata grid), 1 =
+                              the paper's a x 1 row blocks (P:L379, 64 x 1 for Hugewiki; reading
+                              R27): blocks one after another in the order perm(S_STRATA(t), a) */
 } or_params;
 
 typedef struct or_ctx or_ctx;

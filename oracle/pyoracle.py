@@ -44,7 +44,7 @@ class Params(ctypes.Structure):
                 ("batch_f", ctypes.c_int32), ("wf_cols", ctypes.c_int32),
                 ("grid_a", ctypes.c_int32), ("cyclic", ctypes.c_int32),
                 ("lr_rule", ctypes.c_int32), ("ada_eps", ctypes.c_float),
-                ("group_cols", ctypes.c_int32)]
+                ("group_cols", ctypes.c_int32), ("grid_cols", ctypes.c_int32)]
 
 
 _lib = None
@@ -122,7 +122,7 @@ class Oracle:
     def __init__(self, m, n, k, u, v, r, *, lambda_p=0.05, lambda_q=None, alpha=0.08, beta=0.3,
                  init_scale=1.0, rating_scale=1.0, seed=42, schedule="hogwild", storage="fp32",
                  workers=1, batch_f=256, wf_cols=0, grid_a=1, cyclic=False, lr_rule="eq9",
-                 ada_eps=1e-8, group_cols=False):
+                 ada_eps=1e-8, group_cols=False, grid_cols=0):
         self.m, self.n, self.k = int(m), int(n), int(k)
         self.p = Params(m=m, n=n, k=k, lambda_p=lambda_p,
                         lambda_q=lambda_p if lambda_q is None else lambda_q, alpha=alpha,
@@ -130,7 +130,7 @@ class Oracle:
                         schedule=SCHEDULE[schedule], storage=STORAGE[storage], workers=workers,
                         batch_f=batch_f, wf_cols=wf_cols, grid_a=grid_a, cyclic=int(cyclic),
                         lr_rule={"eq9": 0, "adagrad": 1}[lr_rule], ada_eps=ada_eps,
-                        group_cols=int(group_cols))
+                        group_cols=int(group_cols), grid_cols=int(grid_cols))
         self.u = np.ascontiguousarray(u, dtype=np.int32)
         self.v = np.ascontiguousarray(v, dtype=np.int32)
         self.r = np.ascontiguousarray(r, dtype=np.float32)

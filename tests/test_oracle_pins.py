@@ -619,3 +619,67 @@ def test_grouped_batches_permute_within_batches_only():
         assert np.all(np.diff(rho_c[v[perm[seg]]]) >= 0)
         pos += len(batch)
     assert pos == 4000
+
+
+# --------------------------------------------------------------------------- a x 1 row blocks (R27)
+
+def test_row_block_grid_ids_hand_derived(golden_dir):
+    """The paper's a x 1 grid (Hugewiki in 64 x 1 blocks; reading R27): a sample's block
+    is its relabelled row segment alone.  On the App. A case (m = 10, n = 7, a = 2) every cell of
+    row u lands in block row_of_u[u][0] of the hand derivation, whatever its column."""
+    g, cs, o = _grid_case(golden_dir, schedule="hogwild", grid_cols=1)
+    hb = np.empty(cs["N"], np.int64)
+    hb[o.export("perm")] = o.export("blockid")
+    want = [[ru[0]] * cs["n"] for ru in g["row_of_u"]]
+    assert hb.reshape(cs["m"], cs["n"]).tolist() == want
+    # the a x a grid's blocks of row segment r, merged, are the a x 1 block r
+    _, _, oa = _grid_case(golden_dir, schedule="hogwild")
+    ha = np.empty(cs["N"], np.int64)
+    ha[oa.export("perm")] = oa.export("blockid")
+    assert np.array_equal(ha // cs["a"], hb)
+
+
+def test_row_block_epoch_order_hand_derived(golden_dir):
+    """Epoch order of the a x 1 grid: the blocks one after another in the order pi_t =
+    perm(S_STRATA(t), a) of App. A (golden pi_0_a8), each block's chunks in perm(S_HW(t, b))
+    order.  With f larger than any block every block is one chunk, so epoch 0 must visit block
+    pi_0[0]'s samples in storage order, then block pi_0[1]'s, ... (rho_R of the golden)."""
+    ga = golden(golden_dir, "appendix_a.json")
+    m, n, a = 10, 7, 8
+    u = np.repeat(np.arange(m, dtype=np.int32), n)
+    v = np.tile(np.arange(n, dtype=np.int32), m)
+    o = po.Oracle(m, n, 16, u, v, np.ones(m * n, np.float32), seed=ga["seed"], grid_a=a,
+                  grid_cols=1, batch_f=256)
+    rho = ga["rho_R_10"]
+    seg = [rho[uu] * a // m for uu in range(m)]           # floor(a rho / m), A: segments
+    perm = o.export("perm")                                # caller index i = 7u + v per position
+    want = []
+    for b in ga["pi_0_a8"]:
+        want += [p for p in range(m * n) if seg[perm[p] // n] == b]
+    assert o.export("order", 0).tolist() == want
+    assert o.export("strata", 0).tolist() == ga["pi_0_a8"]
+
+
+def test_row_block_grid_with_one_block_is_the_plain_epoch():
+    """a = 1: the a x 1 and a x a grids are the same single block (one Hogwild epoch)."""
+    u, v, r, m, n = _tiny_uniform()
+    o1 = po.Oracle(m, n, 8, u, v, r, grid_a=1, batch_f=32)
+    o2 = po.Oracle(m, n, 8, u, v, r, grid_a=1, grid_cols=1, batch_f=32)
+    for _ in range(2):
+        o1.train_epoch()
+        o2.train_epoch()
+    assert np.array_equal(o1.factors()[0], o2.factors()[0])
+    assert np.array_equal(o1.factors()[1], o2.factors()[1])
+    assert o2.export("order", 3).tolist() == o1.export("order", 3).tolist()
+
+
+def test_row_block_grid_every_sample_once_and_more_blocks_than_columns():
+    """a x 1 needs a <= m only (a may exceed n); every sample is visited once per epoch."""
+    u, v, r, m, n = _tiny_uniform()
+    a = n + 3
+    assert a <= m
+    o = po.Oracle(m, n, 8, u, v, r, grid_a=a, grid_cols=1, batch_f=16)
+    for t in range(2):
+        assert sorted(o.export("order", t).tolist()) == list(range(len(u)))
+    with pytest.raises(Exception):
+        po.Oracle(m, n, 8, u, v, r, grid_a=a)                # a x a still needs a <= n
