@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define MF_ABI_VERSION 4
+#define MF_ABI_VERSION 5
 
 typedef struct mf_ctx mf_ctx; /* opaque, owned by the library */
 
@@ -169,6 +169,14 @@ typedef struct mf_params {
                              mutual exclusion of the ticket protocol on the global P/Q rows,
                              which compute-sanitizer's racecheck (shared memory only) cannot
                              see.  One atomic per wave when on, nothing when off             */
+  int32_t grid_cols;      /* column segments of the grid: 0 = grid_a (the a x a strata grid),
+                             1 = the paper's a x 1 row blocks (Hugewiki in 64 x 1
+                             blocks; reading R27): block r holds the ratings of relabelled row
+                             segment r and all columns, and an epoch trains the a blocks one
+                             after another in the order perm(S_STRATA(t), a), each by batch-
+                             Hogwild.  a <= m (a may exceed n), a <= 256.  One GPU, Hogwild,
+                             Eq. 9 (else MF_E_UNSUPPORTED).  With staged = 2 every P row
+                             segment crosses the host link twice per epoch instead of 2a times */
 } mf_params;
 
 /* Fill *p with defaults (Table 3 Netflix lambda/alpha/beta, k = 128, fp32, Hogwild, f = 256). */

@@ -99,20 +99,22 @@ __global__ void k_rank_of(const uint32_t* __restrict__ perm, int64_t n, int32_t*
 struct Grid {
   int64_t m, n, a, s, c;  // s, c only for wavefront
   bool wf;
+  int64_t ac;             // column segments: a (a x a strata grid) or 1 (a x 1 row blocks, R27)
 };
 
 __device__ __forceinline__ int64_t seg_lo(int64_t r, int64_t a, int64_t n) {
   return cdiv64(r * n, a);
 }
 
-// Bucket of a (relabelled) sample: strata block b = r*a + J, and for the wavefront the
-// sub-block (b*s + i)*c + j inside it (A: "Segments and blocks").
+// Bucket of a (relabelled) sample: strata block b = r*ac + J (ac = a, or 1 for the a x 1 row
+// blocks), and for the wavefront the sub-block (b*s + i)*c + j inside it (A: "Segments and
+// blocks").
 __device__ __forceinline__ uint32_t bucket_of(const Grid& G, int64_t ru, int64_t rc) {
-  const int64_t r = ru * G.a / G.m, J = rc * G.a / G.n;
-  const int64_t b = r * G.a + J;
+  const int64_t r = ru * G.a / G.m, J = rc * G.ac / G.n;
+  const int64_t b = r * G.ac + J;
   if (!G.wf) return (uint32_t)b;
   const int64_t rlo = seg_lo(r, G.a, G.m), rhi = seg_lo(r + 1, G.a, G.m);
-  const int64_t clo = seg_lo(J, G.a, G.n), chi = seg_lo(J + 1, G.a, G.n);
+  const int64_t clo = seg_lo(J, G.ac, G.n), chi = seg_lo(J + 1, G.ac, G.n);
   const int64_t i = (ru - rlo) * G.s / (rhi - rlo);
   const int64_t j = (rc - clo) * G.c / (chi - clo);
   return (uint32_t)((b * G.s + i) * G.c + j);
@@ -512,8 +514,8 @@ float gamma_of(float alpha, float beta, int32_t t) {
 __global__ void k_chunk_records(const int32_t* __restrict__ u, const int32_t* __restrict__ v,
                                 const float* __restrict__ r, int64_t C, int64_t i0, uint64_t S,
                                 const int32_t* __restrict__ rho_r, const int32_t* __restrict__ rho_c,
-                                double rs, int64_t m, int64_t n, int64_t a, int64_t lo_seg,
-                                int64_t hi_seg, uint32_t* __restrict__ blk,
+                                double rs, int64_t m, int64_t n, int64_t a, int64_t ac,
+                                int64_t lo_seg, int64_t hi_seg, uint32_t* __restrict__ blk,
                                 uint32_t* __restrict__ idx, uint64_t* __restrict__ keys,
                                 Rating* __restrict__ recs) {
   for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < C;
@@ -524,7 +526,7 @@ __global__ void k_chunk_records(const int32_t* __restrict__ u, const int32_t* __
     x.r = (float)((double)r[j] / rs);                  // R5, rounded once (as k_build_storage)
     const int64_t seg = (int64_t)x.u * a / m;
     const bool own = seg >= lo_seg && seg < hi_seg;
-    blk[j] = own ? (uint32_t)(seg * a + (int64_t)x.v * a / n) : (uint32_t)(a * a);
+    blk[j] = own ? (uint32_t)(seg * ac + (int64_t)x.v * ac / n) : (uint32_t)(a * ac);
     idx[j] = (uint32_t)j;
     keys[j] = hkey(S, (uint64_t)(i0 + j));              // A: key(S_SHUF, caller index)
     recs[j] = x;
@@ -616,6 +618,7 @@ struct mf_ctx {
 
   int64_t m = 0, n = 0, N = 0, Ntest = 0;
   int k = 0, a = 1, s = 1, c = 1, f = 256, G = 1, rank = 0;
+  int ac = 1;                        // column segments of the grid: a, or 1 (a x 1, R27)
   int32_t t = 0;
   bool wf = false;
 
@@ -1077,8 +1080,13 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
   const int a = p->grid_a > 0 ? p->grid_a : (libmf ? 64 : (world == 1 ? 1 : 8));
-  if (a % world != 0 || a > p->m || a > p->n) return MF_E_INVAL;
-  if (!libmf && (a > 64 || a / world > kMaxSegs)) return MF_E_INVAL;
+  if (p->grid_cols < 0 || p->grid_cols > 1) return MF_E_INVAL;
+  const bool rows_only = p->grid_cols == 1;      // a x 1 row blocks (R27)
+  if (rows_only && (world > 1 || p->schedule != MF_HOGWILD || p->lr_rule != 0))
+    return MF_E_UNSUPPORTED;                     // one GPU, batch-Hogwild, Eq. 9
+  if (a % world != 0 || a > p->m || (!rows_only && a > p->n)) return MF_E_INVAL;
+  if (rows_only && a > 256) return MF_E_INVAL;
+  if (!libmf && !rows_only && (a > 64 || a / world > kMaxSegs)) return MF_E_INVAL;
   if (libmf && a > 1024) return MF_E_INVAL;
   if (p->batch_f < 0 || p->workers < 0 || p->wf_cols < 0) return MF_E_INVAL;
 
@@ -1090,6 +1098,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   c->n = p->n;
   c->k = p->k;
   c->a = a;
+  c->ac = rows_only ? 1 : a;
   c->G = world;
   c->rank = p->rank;
   c->f = p->batch_f > 0 ? p->batch_f : 256;
@@ -1334,7 +1343,7 @@ static mf_status init_factors(mf_ctx* c) {
 }
 
 static mf_status alloc_schedule(mf_ctx* c) {
-  const int64_t nb = (int64_t)c->a * c->a;
+  const int64_t nb = (int64_t)c->a * c->ac;
   int64_t cap = 1;
   if (c->wf) cap = nb * c->s * (int64_t)c->c;
   else cap = c->ch_off.back();
@@ -1429,11 +1438,11 @@ static mf_status setup_staging_buffers(mf_ctx* c) {
   int64_t sum = 0;
   for (int r = c->lo_row_seg(); r < c->hi_row_seg(); ++r) {
     int64_t mx = 0;
-    for (int J = 0; J < c->a; ++J) {
-      const int64_t b = (int64_t)r * c->a + J;
+    for (int J = 0; J < c->ac; ++J) {
+      const int64_t b = (int64_t)r * c->ac + J;
       mx = std::max(mx, c->blk_off[(size_t)b + 1] - c->blk_off[(size_t)b]);
     }
-    sum += mx;
+    sum = c->ac == 1 ? std::max(sum, mx) : sum + mx;   // a x 1: a stratum is one block
   }
   cap = std::max<int64_t>(cap, sum);
   if (c->pq) {                         // one strata block at a time
@@ -1464,9 +1473,11 @@ static mf_status setup_staging_buffers(mf_ctx* c) {
   return MF_OK;
 }
 
-// The blocks this rank trains in sub-epoch j of epoch t (A: strata order).
+// The blocks this rank trains in sub-epoch j of epoch t (A: strata order; a x 1 row blocks,
+// R27: block pi_t[j] alone).
 static std::vector<int64_t> stratum_blocks(const mf_ctx* c, int32_t t, int32_t j) {
   const std::vector<int64_t> pi = host_perm(make_stream(c->p.seed, kTagStrata, (uint64_t)t, 0), c->a);
+  if (c->ac == 1) return std::vector<int64_t>(1, pi[(size_t)j]);
   std::vector<int64_t> out;
   for (int r = c->lo_row_seg(); r < c->hi_row_seg(); ++r)
     out.push_back((int64_t)r * c->a + (r + pi[(size_t)j]) % c->a);
@@ -1619,8 +1630,8 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
   }
 
   // storage-order samples (relabelled, scaled) and their buckets
-  Grid Gd{c->m, c->n, c->a, c->s, c->c, c->wf};
-  const int64_t nb = (int64_t)c->a * c->a;
+  Grid Gd{c->m, c->n, c->a, c->s, c->c, c->wf, c->ac};
+  const int64_t nb = (int64_t)c->a * c->ac;
   const int64_t nbuckets = c->wf ? nb * c->s * (int64_t)c->c : nb;
   Rating* stor = nullptr;
   uint32_t *bk0 = nullptr, *bk1 = nullptr, *pos0 = nullptr, *pos1 = nullptr;
@@ -1793,7 +1804,7 @@ static mf_status load_train(mf_ctx* c, int64_t N, const int32_t* u, const int32_
 // ---------------------------------------------------------------------------------------------
 static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, const int32_t* v,
                                     const float* r) {
-  const int64_t nb = (int64_t)c->a * c->a;
+  const int64_t nb = (int64_t)c->a * c->ac;
   const int64_t C = std::max<int64_t>(
       1, std::min<int64_t>(std::max<int64_t>(N, 1),
                            c->p.stage_chunk > 0 ? c->p.stage_chunk : ((int64_t)1 << 26)));
@@ -1839,7 +1850,7 @@ static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, cons
       if (e != cudaSuccess) { st = c->cuda_fail(e, "chunk validate", __LINE__); break; }
       if (hbad) { st = c->fail(MF_E_RANGE, "rating index out of range or non-finite rating"); break; }
       k_chunk_records<<<g, 256, 0, c->st>>>(cu, cv, cr, n, s0, S, c->rho_r, c->rho_c,
-                                            (double)c->p.rating_scale, c->m, c->n, c->a,
+                                            (double)c->p.rating_scale, c->m, c->n, c->a, c->ac,
                                             c->lo_row_seg(), c->hi_row_seg(), b0, i0, k0, r0);
       if ((e = cudaGetLastError()) != cudaSuccess) { st = c->cuda_fail(e, "k_chunk_records", __LINE__); break; }
       if ((st = c->sort_pairs(b0, b1, i0, i1, n, bits_for((uint64_t)nb))) != MF_OK) break;
@@ -1905,7 +1916,7 @@ static mf_status load_train_chunked(mf_ctx* c, int64_t N, const int32_t* u, cons
   // ---- pass 2
   {
     Nvtx rp2("out-of-core pass 2 (per block)");
-    Grid Gd{c->m, c->n, c->a, c->s, c->c, c->wf};
+    Grid Gd{c->m, c->n, c->a, c->s, c->c, c->wf, c->ac};
     const int64_t per = (int64_t)c->s * c->c;
     uint64_t *k0 = nullptr, *k1 = nullptr;
     uint32_t *i0 = nullptr, *i1 = nullptr, *s0 = nullptr, *s1 = nullptr;
@@ -2148,7 +2159,7 @@ static mf_status join_side(mf_ctx* c) {
 
 static mf_status build_schedule(mf_ctx* c, int32_t t) {
   TRY(join_side(c));
-  const int64_t nb = (int64_t)c->a * c->a;
+  const int64_t nb = (int64_t)c->a * c->ac;
   if (c->libmf) return MF_OK;             // blocks are picked at run time from the table
   if (!c->wf) {
     const int64_t total = c->ch_off.back();
@@ -2505,9 +2516,13 @@ static mf_status train_epoch_strata(mf_ctx* c, int32_t t, float g) {
   for (int j = 0; j < c->a; ++j) {
     Nvtx rj("sub-epoch %d", j);
     int32_t nb = 0, nx = 0;
-    if (mf_strata_plan(c->p.seed, c->a, c->G, c->rank, c->n, t, j, hold, blocks.data(), &nb,
-                       xf.data(), &nx) != MF_OK)
+    if (c->ac == 1) {                  // a x 1 row blocks (R27, one GPU): block pi_t[j]
+      blocks[0] = stratum_blocks(c, t, j)[0];
+      nb = 1;
+    } else if (mf_strata_plan(c->p.seed, c->a, c->G, c->rank, c->n, t, j, hold, blocks.data(), &nb,
+                              xf.data(), &nx) != MF_OK) {
       return c->fail(MF_E_INVAL, "strata plan failed");
+    }
     if (nx) {
       Nvtx rq("Q rotation (%d segments)", nx);
       TRY(rotate_q(c, xf.data(), nx));
@@ -2562,8 +2577,10 @@ static mf_status train_epoch_pq(mf_ctx* c, int32_t t, float g) {
   int64_t x = 0;
   for (int j = 0; j < c->a; ++j) {
     Nvtx rj("sub-epoch %d", j);
-    for (int r = 0; r < c->a; ++r, ++x) {
-      const int64_t b = (int64_t)r * c->a + (r + pi[(size_t)j]) % c->a;
+    for (int rr = 0; rr < (c->ac == 1 ? 1 : c->a); ++rr, ++x) {
+      // a x a: block (r, (r + pi_t[j]) mod a) for every r; a x 1 (R27): block pi_t[j]
+      const int r = c->ac == 1 ? (int)pi[(size_t)j] : rr;
+      const int64_t b = c->ac == 1 ? (int64_t)r : (int64_t)r * c->a + (r + pi[(size_t)j]) % c->a;
       const int s = (int)(x & 1);
       const int64_t lo = cdiv64((int64_t)r * c->m, c->a), hi = cdiv64((int64_t)(r + 1) * c->m, c->a);
       const size_t bytes = (size_t)(hi - lo) * rowb;
@@ -2629,7 +2646,7 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
   }
   CUDA_TRY(c, cudaEventRecord(c->ev_s1, c->st));
   if (c->libmf) {
-    const int64_t nb = (int64_t)c->a * c->a;
+    const int64_t nb = (int64_t)c->a * c->ac;
     const int rem = (int)nb;
     CUDA_TRY(c, cudaMemsetAsync(c->lm_lock, 0, 4, c->st));
     CUDA_TRY(c, cudaMemsetAsync(c->lm_row, 0, (size_t)c->a * 4, c->st));
@@ -2733,7 +2750,7 @@ mf_status mf_check_visits(mf_ctx* c, int64_t* bad_units, int64_t* units, int32_t
   if (c->wf) {
     // a strata block's s*c sub-blocks are visited once per epoch when the rank trains the block
     // (it owns the row segment and the block holds ratings); the others never
-    const int64_t per = (int64_t)c->s * c->c, nb = (int64_t)c->a * c->a;
+    const int64_t per = (int64_t)c->s * c->c, nb = (int64_t)c->a * c->ac;
     for (int64_t b = 0; b < nb; ++b)
       CUDA_TRY(c, launch_visit_check(c->visits + b * per, per, c->blk_len[(size_t)b] > 0 ? e : 0u,
                                      c->chk_dev, c->num_sms, c->st));
@@ -3024,7 +3041,7 @@ mf_status mf_export_schedule(mf_ctx* c, int32_t what, int32_t epoch, int64_t* bu
   if (!c || !len) return MF_E_INVAL;
   TRY(c->enter());
   if (!c->train_loaded) return c->fail(MF_E_STATE, "no train set loaded");
-  const int64_t nb = (int64_t)c->a * c->a;
+  const int64_t nb = (int64_t)c->a * c->ac;
   int64_t need = 0;
   if ((what == MF_EX_PERM && !c->perm) || (what == MF_EX_BLOCKID && !c->slot_pos))
     return c->fail(MF_E_UNSUPPORTED, "per-sample index maps are not kept (staged mode or N > 2^30)");

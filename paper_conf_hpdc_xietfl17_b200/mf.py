@@ -56,7 +56,8 @@ class Params(ctypes.Structure):
                 ("stream", ctypes.c_void_p), ("alloc", ctypes.POINTER(Allocator)),
                 ("launch_blocks", ctypes.c_int32), ("exact_order", ctypes.c_int32),
                 ("rating_stage", ctypes.c_int32), ("stage_chunk", ctypes.c_int64),
-                ("group_cols", ctypes.c_int32), ("check_owners", ctypes.c_int32)]
+                ("group_cols", ctypes.c_int32), ("check_owners", ctypes.c_int32),
+                ("grid_cols", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -221,7 +222,7 @@ class MF:
                  lane_bytes: int = 0, prefetch: int = 0, wf_kernel: int = 0, staged: bool = False,
                  lr_rule: str = "eq9", ada_eps: float = 1e-8, launch_blocks: int = 0,
                  exact_order: bool = False, rating_stage: int = 0, stage_chunk: int = 0,
-                 group_cols: bool = False, check_owners: bool = False,
+                 group_cols: bool = False, check_owners: bool = False, grid_cols: int = 0,
                  device: int = 0, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, transport: int = 0, stream=None,
                  allocator: str = "torch", device_budget: int | None = None):
@@ -243,6 +244,7 @@ class MF:
         p.stage_chunk = int(stage_chunk)
         p.group_cols = int(group_cols)
         p.check_owners = int(check_owners)
+        p.grid_cols = int(grid_cols)
         p.lr_rule, p.ada_eps = {"eq9": 0, "adagrad": 1}[lr_rule], ada_eps
         p.device, p.rank, p.world, p.transport = device, rank, world, transport
         self._id_buf = None

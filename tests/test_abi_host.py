@@ -96,6 +96,9 @@ def test_create_refuses_combinations_no_kernel_implements(L):
     assert refused(rating_stage=1, batch_f=100)                       # f % 64 != 0
     assert refused(group_cols=1, schedule=1)
     assert refused(staged=2, world=2, grid_a=8, rank=0)
+    assert refused(grid_cols=1, grid_a=4, schedule=1)                # a x 1: Hogwild only
+    assert refused(grid_cols=1, grid_a=4, lr_rule=1)
+    assert refused(grid_cols=1, grid_a=8, world=2, rank=0)
 
 
 def test_strata_holders_partition_and_rotation(L):

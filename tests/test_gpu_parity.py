@@ -52,6 +52,7 @@ def ragged():
 INDEX_CASES = [
     dict(schedule="hogwild"),
     dict(schedule="hogwild", batch_f=96, grid_a=8),
+    dict(schedule="hogwild", batch_f=96, grid_a=16, grid_cols=1),               # a x 1 (R27)
     dict(schedule="wavefront", workers=8, wf_cols=16),
     dict(schedule="wavefront", workers=5, wf_cols=7, grid_a=4),
     dict(schedule="wavefront", workers=8, wf_cols=16, cyclic=True),
@@ -746,6 +747,78 @@ def test_out_of_core_load_retried_after_nomem_matches_a_fresh_ctx(staged):
         for Xg, Xw in zip(g.factors(), want):
             assert np.array_equal(Xg, Xw)
         g.close()
+
+
+# ----------------------------------------------------------------------------- a x 1 row blocks
+
+ROW_BLOCK_CASES = [
+    dict(grid_a=4, batch_f=32),
+    dict(grid_a=4, batch_f=32, staged=1),
+    dict(grid_a=4, batch_f=32, staged=1, stage_chunk=1000),
+    dict(grid_a=5, batch_f=32, staged=2),
+    dict(grid_a=5, batch_f=32, staged=2, stage_chunk=777),
+    dict(grid_a=8, batch_f=64, group_cols=True),
+    dict(grid_a=3, batch_f=64, k=128, storage="fp16"),
+    dict(grid_a=250, batch_f=16),                               # a > n (197): rows-only grid
+]
+
+
+@pytest.mark.parametrize("kw", ROW_BLOCK_CASES)
+def test_row_block_grid_matches_the_oracle(kw):
+    """The paper's a x 1 grid (R27): blocks one after another in the order pi_t, each by
+    batch-Hogwild.  At 1 worker: block ids, chunk order and strata order bit-exact, factors
+    within 1e-5 (fp32) / 2e-3 (fp16 values ~0.1-1) of the oracle after 2 epochs, every chunk
+    claimed once; resident, out-of-core ratings and P out of core alike."""
+    kw = dict(kw)
+    k = kw.pop("k", 16)
+    R = ragged()
+    g, o = pair(R, k=k, workers=1, grid_cols=1, seed=5, **TABLE3_NETFLIX, **kw)
+    if not kw.get("staged"):
+        assert np.array_equal(g.export("blockid"), o.export("blockid"))
+    for t in (0, 1):
+        assert np.array_equal(g.export("chunkorder", t), o.export("chunkorder", t))
+        assert np.array_equal(g.export("strata", t), o.export("strata", t))
+    for _ in range(2):
+        g.train_epoch()
+        o.train_epoch()
+        assert g.stats()["updates"] == R.N
+    assert g.check_visits()["bad_units"] == 0
+    tol = 1e-5 if kw.get("storage", "fp32") == "fp32" else 2e-3
+    for Xg, Xo in zip(g.factors(), o.factors()):
+        assert np.abs(Xg - Xo).max() <= tol
+    ro = o.rmse(R.ut, R.vt, R.rt)
+    assert abs(g.rmse() - ro) <= 1e-4 * ro
+    g.close()
+
+
+def test_row_block_grid_full_concurrency_and_p_out_of_core_below_budget():
+    """All resident workers on the a x 1 grid: every chunk claimed once per epoch; with P out of
+    core under a device budget below P's size the run is bit-identical to resident P."""
+    R = synth.uniform(m=40_000, n=600, N=600_000, seed=11, mu=0.5, rank=4, noise=0.1, Ntest=3000)
+    k = 128
+    p_bytes = R.m * k * 4
+    out = []
+    for extra in (dict(), dict(staged=2, stage_chunk=1 << 14, device_budget=p_bytes * 3 // 4)):
+        g = mf.MF(R.m, R.n, k, grid_a=8, grid_cols=1, batch_f=64, workers=1, seed=3,
+                  **TABLE3_NETFLIX, **extra)
+        g.load(R.u, R.v, R.r)
+        g.load(R.ut, R.vt, R.rt, "test")
+        for _ in range(2):
+            g.train_epoch()
+        if extra:
+            assert 0 < g.device_peak_bytes < p_bytes
+        out.append((g.factors(), g.rmse()))
+        g.close()
+    assert np.array_equal(out[0][0][0], out[1][0][0]) and np.array_equal(out[0][0][1], out[1][0][1])
+    assert out[0][1] == out[1][1]
+    g = mf.MF(R.m, R.n, k, grid_a=8, grid_cols=1, batch_f=64, seed=3, **TABLE3_NETFLIX)
+    g.load(R.u, R.v, R.r)
+    for _ in range(3):
+        g.train_epoch()
+        assert g.stats()["updates"] == R.N
+    v = g.check_visits()
+    assert v["bad_units"] == 0 and v["epochs"] == 3
+    g.close()
 
 
 def test_resident_load_fails_cleanly_below_the_device_budget():
