@@ -66,6 +66,8 @@ def parse():
                     help="out-of-core: 1 = ratings in pinned host memory, streamed per stratum; "
                          "2 = P's row segments too, one strata block at a time")
     ap.add_argument("--grid-a", type=int, default=0)
+    ap.add_argument("--grid-cols", type=int, default=0, choices=[0, 1],
+                    help="1 = the paper's a x 1 row blocks (P:L379, reading R27), one GPU")
     ap.add_argument("--lr-rule", default="eq9", choices=["eq9", "adagrad"])
     ap.add_argument("--batch-f", type=int, default=0, help="Eq. 8 f (0 = 256, P:L277)")
     ap.add_argument("--fraction", type=float, default=1.0, help="scale the workload (testing)")
@@ -274,6 +276,11 @@ def cpu_baseline(R, hp, args, sample):
 def resolve_workload(args, world):
     if args.workload is None:
         args.workload = "netflix" if world == 1 else "hugewiki"
+    if world == 1 and args.workload == "hugewiki" and not args.grid_a and not args.grid_cols \
+            and args.schedule == "hogwild" and not args.staged:
+        # one GPU on the Hugewiki shape: the paper's own blocking, i x j = 64 x 1 (
+        # R27).  --grid-a 1 runs the unblocked set.
+        args.grid_a, args.grid_cols = 64, 1
 
 
 def default_f(args, world):
@@ -343,7 +350,9 @@ def config_of(args, R, world):
             "fraction": args.fraction, "exact_order": bool(args.exact_order),
             "rating_stage": "tma" if args.rating_stage else "lane-loads",
             "group_cols": bool(args.group_cols),
-            "staged": int(args.staged), "grid_a": args.grid_a or (8 if world > 1 else 1),
+            "staged": int(args.staged),
+            "grid_a": getattr(args, "grid_a_used", None) or args.grid_a or (8 if world > 1 else 1),
+            "grid": "a x 1 row blocks" if args.grid_cols == 1 else "a x a strata",
             "l2": "inputs larger than L2 (COO %.2f GB per epoch); model P+Q stays cached as in "
                   "any training run" % (R.N * 12 / 1e9)}
 
@@ -356,11 +365,15 @@ def ncu_traffic(args):
         return None, None
     with open(path) as f:
         d = json.load(f)
+    a_used = getattr(args, "grid_a_used", None) or args.grid_a or 1
     key = f"{args.workload}/{args.schedule}/{args.storage}/k{args.k}"
+    if args.grid_cols:
+        key += f"/rows{a_used}"
     e = d.get(key, {})
     # a capture describes one launch configuration: plain or grouped batches of f, full size
     if (e.get("batch_f", 256) != default_f(args, 1) or e.get("group_cols", False) != bool(args.group_cols)
-            or e.get("fraction", 1.0) != args.fraction):
+            or e.get("fraction", 1.0) != args.fraction or e.get("grid_cols", 0) != args.grid_cols
+            or e.get("grid_a", 1) != a_used):
         return None, None
     return e.get("dram_bytes_per_launch"), e.get("source")
 
@@ -380,6 +393,7 @@ def rank_main(args, C, R=None, out=None):
     kw = dict(schedule=args.schedule, storage=args.storage, workers=args.workers,
               wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes,
               prefetch=args.prefetch, wf_kernel=args.wf_kernel, grid_a=args.grid_a,
+              grid_cols=args.grid_cols,
               batch_f=default_f(args, world), lr_rule=args.lr_rule, seed=42,
               exact_order=args.exact_order, rating_stage=args.rating_stage,
               group_cols=args.group_cols, device=C.local, rank=rank, world=world,
@@ -393,6 +407,7 @@ def rank_main(args, C, R=None, out=None):
     model.load(R.u, R.v, R.r, "train")
     model.load(R.ut, R.vt, R.rt, "test")
     rmse0 = model.rmse("test")
+    args.grid_a_used = int(len(model.export("strata", 0)))     # a x 1 with grid_a = 0: auto
 
     for _ in range(args.warmup):
         model.train_epoch()
@@ -442,20 +457,28 @@ def rank_main(args, C, R=None, out=None):
         dram = traffic / (avg_launch_ms / 1000.0) / 1e9
         roof["dram"] = {"achieved": dram, "frac": dram / hbm, "traffic_source": tsrc,
                         "traffic_over_algorithmic": traffic / per_launch_bytes,
-                        "limiter": "hot q_v rows (L2 read-modify-write rate of the power-law-hot "
-                                   "columns, profiles/r01_scaling_hot_rows.md) on Netflix; DRAM on "
-                                   "Yahoo (profiles/r01g_yahoo_fp16_hogwild.md)"}
+                        "limiter": ("a x 1 row blocks: the block's P segment and Q stay in L2, "
+                                    "DRAM carries little more than the ratings; L2 latency and the "
+                                    "hot q_v rows bound it (profiles/r02_row_blocks.md)")
+                                   if args.grid_cols else
+                                   ("hot q_v rows (L2 read-modify-write rate of the power-law-hot "
+                                    "columns, profiles/r01_scaling_hot_rows.md) on Netflix; DRAM on "
+                                    "Yahoo (profiles/r01g_yahoo_fp16_hogwild.md)")}
     model.close()
     del model
 
     e2e = None
     if not args.no_e2e and not (big and world == 1):
         e2e = run_e2e(args, R, kw, stream, C)
-    det = grp = None
+    det = grp = rowb = None
     if not args.no_deterministic and world == 1 and args.schedule == "hogwild" and not big:
         det = run_deterministic(args, R, hp, stream)
         if not args.group_cols:
-            grp = run_grouped(args, R, hp, stream)
+            grp = run_variant(args, R, hp, stream, "hogwild, column-grouped batches (R24), f=1024",
+                              group_cols=True, batch_f=1024)
+        if not args.grid_cols:
+            rowb = run_variant(args, R, hp, stream, "hogwild on the a x 1 row-block grid (R27)",
+                               grid_cols=1)
     cpu = None
     if not args.no_cpu_baseline and rank == 0:
         cpu = cpu_baseline(R, hp, args, args.cpu_sample)
@@ -476,6 +499,7 @@ def rank_main(args, C, R=None, out=None):
                              "epochs": visits["epochs"], "updates_per_epoch": all_updates / args.steps,
                              "N": R.N},
             "e2e": e2e, "cpu_baseline": cpu, "deterministic": det, "grouped": grp,
+            "row_blocks": rowb,
             "paper_context": "cuMF_SGD Table 5 (P:L414-415), fp16 Hogwild: Netflix 267M/s TITAN X, "
                              "613M/s P100; Hugewiki 256M/s / 710M/s (other hardware; context only)"}
     if isinstance(C, ThreadRank):
@@ -529,13 +553,16 @@ def run_deterministic(args, R, hp, stream):
     return out
 
 
-def run_grouped(args, R, hp, stream):
-    """The same Hogwild run with column-grouped batches (reading R24, params.group_cols) at
-    f = 1024 (profiles/r02_grouped_batches.md): device-timed like the main line, same data."""
+def run_variant(args, R, hp, stream, label, **variant):
+    """The same Hogwild run in another of the method's configurations, device-timed like the
+    main line, on the same data: `grouped` = column-grouped batches (reading R24,
+    params.group_cols) at f = 1024 (profiles/r02_grouped_batches.md); `row_blocks` = the paper's
+    a x 1 row-block grid (reading R27; params.grid_cols = 1, a picked so that a P row
+    segment is ~32 MiB: profiles/r02_row_blocks.md)."""
     from paper_conf_hpdc_xietfl17_b200 import mf
     steps, warm = max(3, args.steps // 2), 3
     m = mf.MF(R.m, R.n, args.k, stream=stream, schedule="hogwild", storage=args.storage,
-              group_cols=True, batch_f=1024, seed=42, **hp)
+              seed=42, **hp, **variant)
     m.load(R.u, R.v, R.r, "train")
     m.load(R.ut, R.vt, R.rt, "test")
     for _ in range(warm):
@@ -556,12 +583,15 @@ def run_grouped(args, R, hp, stream):
     hbm, _ = peaks()
     bpu = st["bytes_per_update"]
     achieved = upd * bpu / (float(np.sum(sgd)) / 1000.0) / 1e9
-    out = {"schedule": "hogwild, column-grouped batches (R24), f=1024", "storage": args.storage,
+    out = {"schedule": label, "storage": args.storage,
            "value": upd / (ms / 1000.0), "unit": "updates/s", "ms_per_step": ms / steps,
            "steps": steps, "warmup": warm, "test_rmse": m.rmse("test"),
            "exactly_once_bad_units": m.check_visits()["bad_units"],
+           "sgd_launches_per_epoch": st["sgd_launches"],
            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                         "frac": achieved / hbm, "bytes_per_update": bpu}}
+    if variant.get("grid_cols"):
+        out["grid_a"] = int(len(m.export("strata", 0)))
     m.close()
     return out
 

@@ -174,7 +174,9 @@ typedef struct mf_params {
                              blocks; reading R27): block r holds the ratings of relabelled row
                              segment r and all columns, and an epoch trains the a blocks one
                              after another in the order perm(S_STRATA(t), a), each by batch-
-                             Hogwild.  a <= m (a may exceed n), a <= 256.  One GPU, Hogwild,
+                             Hogwild.  a <= m (a may exceed n), a <= 256; grid_a = 0 picks a
+                             = ceil(|P| / 32 MiB) (a segment of P stays L2-resident while its
+                             block trains: Netflix 4, Yahoo 8, Hugewiki 256).  One GPU, Hogwild,
                              Eq. 9 (else MF_E_UNSUPPORTED).  With staged = 2 every P row
                              segment crosses the host link twice per epoch instead of 2a times */
 } mf_params;

@@ -1079,9 +1079,16 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   if (p->lr_rule == 1 && p->schedule == MF_LIBMF) return MF_E_UNSUPPORTED;
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
-  const int a = p->grid_a > 0 ? p->grid_a : (libmf ? 64 : (world == 1 ? 1 : 8));
   if (p->grid_cols < 0 || p->grid_cols > 1) return MF_E_INVAL;
   const bool rows_only = p->grid_cols == 1;      // a x 1 row blocks (R27)
+  // a x 1 with grid_a = 0: blocks whose P row segment is ~32 MiB, a fraction of the 126-MB L2
+  // (profiles/r02_row_blocks.md)
+  const int64_t seg_target = (int64_t)32 << 20;
+  const int64_t p_bytes = p->m * (int64_t)p->k * (p->storage == MF_FP32 ? 4 : 2);
+  const int a = p->grid_a > 0 ? p->grid_a
+                : rows_only ? (int)std::max<int64_t>(1, std::min<int64_t>(std::min<int64_t>(256, p->m),
+                                                                         cdiv64(p_bytes, seg_target)))
+                : (libmf ? 64 : (world == 1 ? 1 : 8));
   if (rows_only && (world > 1 || p->schedule != MF_HOGWILD || p->lr_rule != 0))
     return MF_E_UNSUPPORTED;                     // one GPU, batch-Hogwild, Eq. 9
   if (a % world != 0 || a > p->m || (!rows_only && a > p->n)) return MF_E_INVAL;

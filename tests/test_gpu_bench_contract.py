@@ -41,6 +41,17 @@ def test_bench_json_line_contract():
     cb = d["cpu_baseline"]
     assert cb["kind"] == "oracle" and cb["cores"] == 1 and cb["value"] > 0
     assert d["deterministic"]["roofline"]["frac"] > 0
+    for extra in ("grouped", "row_blocks"):
+        assert d[extra]["value"] > 0 and d[extra]["exactly_once_bad_units"] == 0, extra
+    assert d["row_blocks"]["grid_a"] >= 1
+
+
+def test_bench_hugewiki_one_gpu_uses_the_papers_64x1_blocks():
+    """--workload hugewiki at N = 1 runs the paper's own blocking (i x j = 64 x 1)."""
+    d = _bench("--workload", "hugewiki", "--steps", "3", "--warmup", "3", "--fraction", "0.01",
+               "--no-e2e", "--cpu-sample", "20000", "--no-deterministic")
+    assert d["config"]["grid_a"] == 64 and d["config"]["grid"] == "a x 1 row blocks"
+    assert d["exactly_once"]["bad_units"] == 0 and d["value"] > 0
 
 
 def test_bench_reference_arm_line():

@@ -1,5 +1,5 @@
 """Print the 20-epoch test RMSE of the bench configuration (fp16 Hogwild, all resident workers),
-the grouped-batch variant and the fp16 deterministic wavefront on the full Netflix-shaped set,
+the grouped-batch and a x 1 row-block variants and the fp16 deterministic wavefront on the full Netflix-shaped set,
 next to the oracle's own 20-epoch run (tests/golden/netflix_oracle_fp16_hogwild_k128_e20.json)."""
 import json
 import os
@@ -16,6 +16,8 @@ gold = json.load(open(os.path.join(ROOT, "tests", "golden", "netflix_oracle_fp16
 print("checksum", synth.checksum(R), "golden", gold["data_checksum"])
 runs = {"hogwild": dict(schedule="hogwild"),
         "hogwild-grouped-f1024": dict(schedule="hogwild", group_cols=True, batch_f=1024),
+        "hogwild-rowblocks-auto": dict(schedule="hogwild", grid_cols=1),
+        "hogwild-rowblocks-2x1": dict(schedule="hogwild", grid_cols=1, grid_a=2),
         "wavefront-fp16-cyclic": dict(schedule="wavefront", workers=888, wf_cols=7680, cyclic=True)}
 out = {}
 for name, kw in runs.items():
