@@ -645,6 +645,7 @@ struct mf_ctx {
   // Hogwild: the next epoch's chunk order is built on a side stream (ss) into chunk_order_alt
   // while this epoch's SGD kernel runs (its sorts fill the SMs its retiring blocks free).
   uint32_t* chunk_order_alt = nullptr;
+  uint32_t* chunk_seq = nullptr;     // a x 1 resident: the epoch's chunk ids, blocks in pi_t order
   cudaStream_t ss = nullptr;
   cudaEvent_t ev_ss_go = nullptr, ev_ss_done = nullptr;
   int32_t prebuilt_t = -1;           // epoch whose order chunk_order_alt holds (-1: none)
@@ -818,7 +819,7 @@ struct mf_ctx {
         (void**)&slots, (void**)&slot_pos, (void**)&perm, (void**)&rho_r, (void**)&rho_c, &P, &Q,
         (void**)&test, (void**)&dup, (void**)&sub_off, (void**)&d_choff, (void**)&sk0,
         (void**)&sk1, (void**)&sv0, (void**)&sv1, (void**)&sb, (void**)&chunk_order,
-        (void**)&chunk_order_alt, (void**)&seq, (void**)&rank_arr, (void**)&tickets,
+        (void**)&chunk_order_alt, (void**)&chunk_seq, (void**)&seq, (void**)&rank_arr, (void**)&tickets,
         (void**)&tau, (void**)&sigma, &tmp, (void**)&GP, (void**)&GQ, (void**)&d_blk_off,
         (void**)&d_blk_len, (void**)&lm_lock, (void**)&lm_row, (void**)&lm_col, (void**)&lm_done,
         (void**)&lm_rem, (void**)&stg[0], (void**)&stg[1], (void**)&stg_dup[0],
@@ -1380,6 +1381,7 @@ static mf_status alloc_schedule(mf_ctx* c) {
   } else {
     TRY(c->alloc(&c->chunk_order, (size_t)cap));
     TRY(c->alloc(&c->chunk_order_alt, (size_t)cap));
+    if (c->ac == 1 && !c->staged) TRY(c->alloc(&c->chunk_seq, (size_t)cap));
   }
   return MF_OK;
 }
@@ -2304,6 +2306,35 @@ static void finalize_segs(ChunkSegs& s) {
   for (int l = s.nlev + 1; l <= kMaxSegs; ++l) s.lev_base[l] = base;
 }
 
+// One Hogwild launch over the claim order `segs` of the chunk-id list `chunks`.
+static mf_status launch_chunks(mf_ctx* c, ChunkSegs& segs, const uint32_t* chunks, const Rating* slots,
+                               float g) {
+  finalize_segs(segs);
+  CUDA_TRY(c, cudaMemsetAsync(c->counter, 0, sizeof(unsigned long long), c->st));
+  {
+    HogwildLaunch L{};
+    L.storage = c->p.storage; L.k = c->k; L.lane_bytes = c->p.lane_bytes ? c->p.lane_bytes : 16;
+    L.prefetch = c->p.prefetch ? c->p.prefetch : 1;
+    L.rating_stage = c->p.rating_stage;
+    L.group = c->p.group_cols;
+    L.slots = slots; L.chunks = chunks; L.segs = segs; L.counter = c->counter;
+    L.workers = c->p.workers; L.num_sms = c->num_sms; L.f = c->f;
+    L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
+    L.ada = ada_args(c);
+    L.exact = c->p.exact_order;
+    if (L.ada.GP) L.g = c->p.alpha;        // ADAGRAD: constant alpha, no Eq. 9 decay
+    L.out_workers = &c->last_workers; L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
+    L.visits = c->visits; L.upd = c->upd_dev;
+    CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
+    CUDA_TRY(c, launch_hogwild(L));
+    CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd + 1), c->st));
+    c->last_block = 256;
+    ++c->n_sgd;
+    ++c->n_launch;
+  }
+  return MF_OK;
+}
+
 static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, float g, int buf) {
   const Rating* slots = c->staged ? c->stg[buf] : c->slots;
   const uint16_t* dup = c->staged ? c->stg_dup[buf] : c->dup;
@@ -2320,28 +2351,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
       ++segs.n;
     }
     if (segs.n == 0) return MF_OK;
-    finalize_segs(segs);
-    CUDA_TRY(c, cudaMemsetAsync(c->counter, 0, sizeof(unsigned long long), c->st));
-    HogwildLaunch L{};
-    L.storage = c->p.storage; L.k = c->k; L.lane_bytes = c->p.lane_bytes ? c->p.lane_bytes : 16;
-    L.prefetch = c->p.prefetch ? c->p.prefetch : 1;
-    L.rating_stage = c->p.rating_stage;
-    L.group = c->p.group_cols;
-    L.slots = slots; L.chunks = c->chunk_order; L.segs = segs; L.counter = c->counter;
-    L.workers = c->p.workers; L.num_sms = c->num_sms; L.f = c->f;
-    L.P = c->P; L.Q = c->Q; L.g = g; L.lp = c->p.lambda_p; L.lq = c->p.lambda_q; L.stream = c->st;
-    L.ada = ada_args(c);
-    L.exact = c->p.exact_order;
-    if (L.ada.GP) L.g = c->p.alpha;        // ADAGRAD: constant alpha, no Eq. 9 decay
-    L.out_workers = &c->last_workers; L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
-    L.visits = c->visits; L.upd = c->upd_dev;
-    CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
-    CUDA_TRY(c, launch_hogwild(L));
-    CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd + 1), c->st));
-    c->last_block = 256;
-    ++c->n_sgd;
-    ++c->n_launch;
-    return MF_OK;
+    return launch_chunks(c, segs, c->chunk_order, slots, g);
   }
   // The non-empty blocks run together in one cooperative launch (they touch disjoint rows and
   // columns, so any concurrency gives the result of running them one after another): worker w
@@ -2568,6 +2578,33 @@ static mf_status train_epoch_strata(mf_ctx* c, int32_t t, float g) {
   return MF_OK;
 }
 
+// a x 1 row blocks, resident (R27): the blocks' chunk orders concatenated in pi_t order and run
+// by ONE Hogwild launch -- the claim order is block pi_t[0]'s chunks, then pi_t[1]'s, ..., so a
+// single worker runs exactly the oracle's block-after-block order, and many workers overlap
+// consecutive blocks only at their boundary instead of idling in a per-block tail.
+static mf_status train_epoch_rows(mf_ctx* c, int32_t t, float g) {
+  const std::vector<int64_t> pi = host_perm(make_stream(c->p.seed, kTagStrata, (uint64_t)t, 0), c->a);
+  int64_t off = 0;
+  for (int j = 0; j < c->a; ++j) {
+    const int64_t b = pi[(size_t)j];
+    const int64_t lo = c->ch_off[(size_t)b], nch = c->ch_off[(size_t)b + 1] - lo;
+    if (nch == 0) continue;
+    CUDA_TRY(c, cudaMemcpyAsync(c->chunk_seq + off, c->chunk_order + lo, (size_t)nch * 4,
+                                cudaMemcpyDeviceToDevice, c->st));
+    off += nch;
+  }
+  CUDA_TRY(c, cudaEventRecord(c->ev_c0, c->st));
+  CUDA_TRY(c, cudaEventRecord(c->ev_c1, c->st));
+  if (off == 0) return MF_OK;
+  ChunkSegs segs{};
+  segs.n = 1;
+  segs.begin[0] = 0;
+  segs.prefix[0] = 0;
+  segs.prefix[1] = off;
+  segs.shift[0] = 0;
+  return launch_chunks(c, segs, c->chunk_seq, c->slots, g);
+}
+
 // staged == 2 (section 6.1 step 3 + 6.3): blocks one at a time in the strata order, each with
 // its P row segment staged in on the copy stream, trained on the compute stream, written back on
 // the write-back stream; the next block's copy-in overlaps this block's compute, and its
@@ -2685,7 +2722,8 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
     if (epoch_done) *epoch_done = c->t;
     return MF_OK;
   }
-  TRY(c->pq ? train_epoch_pq(c, t, g) : train_epoch_strata(c, t, g));
+  TRY(c->pq ? train_epoch_pq(c, t, g)
+             : (c->ac == 1 && !c->staged) ? train_epoch_rows(c, t, g) : train_epoch_strata(c, t, g));
   CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
   if (hog) TRY(prebuild_schedule(c, t + 1));   // enqueued after this epoch's SGD launches
   c->t = t + 1;
