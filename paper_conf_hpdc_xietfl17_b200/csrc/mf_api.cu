@@ -1350,6 +1350,13 @@ static mf_status init_factors(mf_ctx* c) {
   return MF_OK;
 }
 
+// a x 1 row blocks (R27) with a > 1, Hogwild, resident: the epoch is one launch over the blocks'
+// concatenated chunk orders (train_epoch_rows).  The 1 x 1 grid (ac == 1 as well) and the
+// wavefront keep the per-stratum path.
+static bool rows_one_launch(const mf_ctx* c) {
+  return !c->wf && c->ac == 1 && c->a > 1 && !c->staged;
+}
+
 static mf_status alloc_schedule(mf_ctx* c) {
   const int64_t nb = (int64_t)c->a * c->ac;
   int64_t cap = 1;
@@ -1381,7 +1388,7 @@ static mf_status alloc_schedule(mf_ctx* c) {
   } else {
     TRY(c->alloc(&c->chunk_order, (size_t)cap));
     TRY(c->alloc(&c->chunk_order_alt, (size_t)cap));
-    if (c->ac == 1 && !c->staged) TRY(c->alloc(&c->chunk_seq, (size_t)cap));
+    if (rows_one_launch(c)) TRY(c->alloc(&c->chunk_seq, (size_t)cap));
   }
   return MF_OK;
 }
@@ -2723,7 +2730,7 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
     return MF_OK;
   }
   TRY(c->pq ? train_epoch_pq(c, t, g)
-             : (c->ac == 1 && !c->staged) ? train_epoch_rows(c, t, g) : train_epoch_strata(c, t, g));
+             : rows_one_launch(c) ? train_epoch_rows(c, t, g) : train_epoch_strata(c, t, g));
   CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
   if (hog) TRY(prebuild_schedule(c, t + 1));   // enqueued after this epoch's SGD launches
   c->t = t + 1;
