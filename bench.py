@@ -68,6 +68,9 @@ def parse():
     ap.add_argument("--grid-a", type=int, default=0)
     ap.add_argument("--grid-cols", type=int, default=0, choices=[0, 1],
                     help="1 = the paper's a x 1 row blocks (P:L379, reading R27), one GPU")
+    ap.add_argument("--q-cache", type=int, default=0, choices=[0, 1],
+                    help="q_v row loads: 0 = through L1 where the Hogwild kernel has it (reading R28), "
+                         "1 = L2 only (params.q_cache)")
     ap.add_argument("--lr-rule", default="eq9", choices=["eq9", "adagrad"])
     ap.add_argument("--batch-f", type=int, default=0, help="Eq. 8 f (0 = 256, P:L277)")
     ap.add_argument("--fraction", type=float, default=1.0, help="scale the workload (testing)")
@@ -353,6 +356,7 @@ def config_of(args, R, world):
             "staged": int(args.staged),
             "grid_a": getattr(args, "grid_a_used", None) or args.grid_a or (8 if world > 1 else 1),
             "grid": "a x 1 row blocks" if args.grid_cols == 1 else "a x a strata",
+            "q_loads": getattr(args, "q_loads_used", None),
             "l2": "inputs larger than L2 (COO %.2f GB per epoch); model P+Q stays cached as in "
                   "any training run" % (R.N * 12 / 1e9)}
 
@@ -369,11 +373,13 @@ def ncu_traffic(args):
     key = f"{args.workload}/{args.schedule}/{args.storage}/k{args.k}"
     if args.grid_cols:
         key += f"/rows{a_used}"
+    if args.schedule == "hogwild" and args.q_cache == 0:
+        key += "/qL1"
     e = d.get(key, {})
     # a capture describes one launch configuration: plain or grouped batches of f, full size
     if (e.get("batch_f", 256) != default_f(args, 1) or e.get("group_cols", False) != bool(args.group_cols)
             or e.get("fraction", 1.0) != args.fraction or e.get("grid_cols", 0) != args.grid_cols
-            or e.get("grid_a", 1) != a_used):
+            or e.get("grid_a", 1) != a_used or e.get("q_cache", 1) != args.q_cache):
         return None, None
     return e.get("dram_bytes_per_launch"), e.get("source")
 
@@ -393,7 +399,7 @@ def rank_main(args, C, R=None, out=None):
     kw = dict(schedule=args.schedule, storage=args.storage, workers=args.workers,
               wf_cols=args.wf_cols, cyclic=args.cyclic, lane_bytes=args.lane_bytes,
               prefetch=args.prefetch, wf_kernel=args.wf_kernel, grid_a=args.grid_a,
-              grid_cols=args.grid_cols,
+              grid_cols=args.grid_cols, q_cache=args.q_cache,
               batch_f=default_f(args, world), lr_rule=args.lr_rule, seed=42,
               exact_order=args.exact_order, rating_stage=args.rating_stage,
               group_cols=args.group_cols, device=C.local, rank=rank, world=world,
@@ -412,6 +418,8 @@ def rank_main(args, C, R=None, out=None):
     for _ in range(args.warmup):
         model.train_epoch()
     torch.cuda.synchronize()
+    if args.schedule == "hogwild" and args.warmup:
+        args.q_loads_used = ("L1 (ld.ca; reading R28)" if model.stats()["q_l1"] else "L2 (.cg)")
     C.barrier()
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
@@ -470,15 +478,19 @@ def rank_main(args, C, R=None, out=None):
     e2e = None
     if not args.no_e2e and not (big and world == 1):
         e2e = run_e2e(args, R, kw, stream, C)
-    det = grp = rowb = None
+    det = grp = rowb = ql2 = None
     if not args.no_deterministic and world == 1 and args.schedule == "hogwild" and not big:
         det = run_deterministic(args, R, hp, stream)
         if not args.group_cols:
             grp = run_variant(args, R, hp, stream, "hogwild, column-grouped batches (R24), f=1024",
-                              group_cols=True, batch_f=1024)
+                              group_cols=True, batch_f=1024, q_cache=args.q_cache)
         if not args.grid_cols:
             rowb = run_variant(args, R, hp, stream, "hogwild on the a x 1 row-block grid (R27)",
-                               grid_cols=1)
+                               grid_cols=1, q_cache=args.q_cache)
+        if args.q_cache == 0:
+            ql2 = run_variant(args, R, hp, stream, "hogwild, q_v loads through L2 only (q_cache = 1)",
+                              q_cache=1, group_cols=bool(args.group_cols),
+                              batch_f=default_f(args, world), grid_cols=args.grid_cols)
     cpu = None
     if not args.no_cpu_baseline and rank == 0:
         cpu = cpu_baseline(R, hp, args, args.cpu_sample)
@@ -499,7 +511,7 @@ def rank_main(args, C, R=None, out=None):
                              "epochs": visits["epochs"], "updates_per_epoch": all_updates / args.steps,
                              "N": R.N},
             "e2e": e2e, "cpu_baseline": cpu, "deterministic": det, "grouped": grp,
-            "row_blocks": rowb,
+            "row_blocks": rowb, "q_l2_only": ql2,
             "paper_context": "cuMF_SGD Table 5 (P:L414-415), fp16 Hogwild: Netflix 267M/s TITAN X, "
                              "613M/s P100; Hugewiki 256M/s / 710M/s (other hardware; context only)"}
     if isinstance(C, ThreadRank):

@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define MF_ABI_VERSION 5
+#define MF_ABI_VERSION 6
 
 typedef struct mf_ctx mf_ctx; /* opaque, owned by the library */
 
@@ -179,6 +179,18 @@ typedef struct mf_params {
                              block trains: Netflix 4, Yahoo 8, Hugewiki 256).  One GPU, Hogwild,
                              Eq. 9 (else MF_E_UNSUPPORTED).  With staged = 2 every P row
                              segment crosses the host link twice per epoch instead of 2a times */
+  int32_t q_cache;        /* batch-Hogwild: cache policy of the q_v row loads (reading R28; the
+                             per-instruction "cache or bypass" choice of section 4, P:L234,
+                             made for the feature row with temporal reuse).  0 = auto: q_v rows
+                             are read through the SM's L1 (ld.ca, write-back stores) in the
+                             Hogwild kernels with >= 16-B lanes on the Eq. 9 fast-form path
+                             (plain and column-grouped batches): a hot column is then read from
+                             L1 by every worker of the SM instead of by an L2 load that
+                             serialises with other SMs' stores to the same line.  L1 is not
+                             coherent across SMs, so a read may miss other SMs' latest store --
+                             a racy read, which Hogwild permits (R19).  Every other kernel and
+                             path reads through L2.  1 = L2 only (.cg loads, .cg stores)
+                             everywhere.  mf_stats.q_l1 reports which one ran                 */
 } mf_params;
 
 /* Fill *p with defaults (Table 3 Netflix lambda/alpha/beta, k = 128, fp32, Hogwild, f = 256). */
@@ -261,6 +273,7 @@ typedef struct mf_stats {
                                (9 or 10 per rating packed, see params.staged; 12 unpacked; +2
                                with the wavefront's duplicate distances; + P's row segments
                                when staged = 2)                                                 */
+  int32_t q_l1;             /* 1 if the last SGD launch read q_v rows through L1 (q_cache) */
 } mf_stats;
 mf_status mf_get_stats(mf_ctx* ctx, mf_stats* out);
 

@@ -674,7 +674,7 @@ struct mf_ctx {
   cudaEvent_t ev_e0 = nullptr, ev_e1 = nullptr, ev_s0 = nullptr, ev_s1 = nullptr;
   cudaEvent_t ev_c0 = nullptr, ev_c1 = nullptr;
   int n_sgd = 0, n_launch = 0;
-  int last_workers = 0, last_lanes = 0, last_grid = 0, last_block = 0;
+  int last_workers = 0, last_lanes = 0, last_grid = 0, last_block = 0, last_q_l1 = 0;
   bool have_stats = false;
   std::vector<double> comm_ms_acc;
 
@@ -1081,6 +1081,7 @@ mf_status mf_create(const mf_params* p, mf_ctx** out) {
   const int world = p->world > 0 ? p->world : 1;
   if (p->rank < 0 || p->rank >= world) return MF_E_INVAL;
   if (p->grid_cols < 0 || p->grid_cols > 1) return MF_E_INVAL;
+  if (p->q_cache < 0 || p->q_cache > 1) return MF_E_INVAL;
   const bool rows_only = p->grid_cols == 1;      // a x 1 row blocks (R27)
   // a x 1 with grid_a = 0: blocks whose P row segment is ~32 MiB, a fraction of the 126-MB L2
   // (profiles/r02_row_blocks.md)
@@ -2331,6 +2332,7 @@ static mf_status launch_chunks(mf_ctx* c, ChunkSegs& segs, const uint32_t* chunk
     L.exact = c->p.exact_order;
     if (L.ada.GP) L.g = c->p.alpha;        // ADAGRAD: constant alpha, no Eq. 9 decay
     L.out_workers = &c->last_workers; L.out_lanes = &c->last_lanes; L.out_grid = &c->last_grid;
+    L.q_l1 = c->p.q_cache == 0; L.out_q_l1 = &c->last_q_l1;
     L.visits = c->visits; L.upd = c->upd_dev;
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd), c->st));
     CUDA_TRY(c, launch_hogwild(L));
@@ -2442,6 +2444,7 @@ static mf_status run_stratum(mf_ctx* c, const std::vector<int64_t>& blocks, floa
     CUDA_TRY(c, e);
     CUDA_TRY(c, cudaEventRecord(ev_at(c, 2 * c->n_sgd + 1), c->st));
     c->last_workers = nw;
+    c->last_q_l1 = 0;
     c->last_block = 128;
     ++c->n_sgd;
     ++c->n_launch;
@@ -2720,6 +2723,7 @@ mf_status mf_train_epoch(mf_ctx* c, int32_t* epoch_done) {
     c->n_sgd = 1;
     c->n_launch += 1;
     c->last_workers = L.workers;
+    c->last_q_l1 = 0;
     c->last_grid = L.workers;
     c->last_block = 32;
     CUDA_TRY(c, cudaEventRecord(c->ev_e1, c->st));
@@ -2788,6 +2792,7 @@ mf_status mf_get_stats(mf_ctx* c, mf_stats* out) {
   out->h2d_bytes = c->h2d_bytes;
   out->workers = c->last_workers;
   out->lanes = c->last_lanes;
+  out->q_l1 = c->last_q_l1;
   out->grid = c->last_grid;
   out->block = c->last_block;
   return MF_OK;

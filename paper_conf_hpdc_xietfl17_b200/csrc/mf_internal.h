@@ -34,6 +34,7 @@ struct HogwildLaunch {
   int storage, k, lane_bytes, prefetch;
   int rating_stage;         // 0 = per-lane streaming loads + shuffles, 1 = TMA bulk copies
   int group;                // params.group_cols: column-grouped batches (R24)
+  int q_l1;                 // params.q_cache == 0: q_v loads through L1 where the kernel has it (R28)
   const Rating* slots;
   const uint32_t* chunks;
   ChunkSegs segs;
@@ -47,6 +48,7 @@ struct HogwildLaunch {
   unsigned long long* upd;  // non-sentinel samples updated (device count, Eq. 7)
   cudaStream_t stream;
   int *out_workers, *out_lanes, *out_grid;
+  int* out_q_l1;            // 1 if the launched kernel read q_v through L1
 };
 
 // The strata blocks one wavefront launch runs concurrently (a stratum's blocks touch disjoint

@@ -32,10 +32,16 @@ constexpr bool narrow16_ring(int K, int S) { return K * S == 64; }
 // 5 resident blocks (40 warps) per SM: 48 registers, a few bytes of stack.  Yahoo-shaped
 // (DRAM-bound) 34.9 -> 33.8 ms/epoch against 4 blocks at 64 registers, Netflix unchanged (hot
 // rows); the ADAGRAD, depth-2 and 32-B-per-lane variants keep the compiler's choice.
+// LC: cache policy of the Hogwild row accesses (bit 0: q_v loads via L1, bit 1: p_u loads via
+// L1, bit 2: q_v stores .wb, bit 3: p_u stores .wb).  0 = L2 only (.cg); kLcQ = q_v through L1
+// (params.q_cache = 0, reading R28).  Measured on B200 (profiles/r02_q_l1.md): q_v via L1 is
+// Netflix fp16 13.99 -> 11.63 ms, k = 32 9.09 -> 7.16 ms, Yahoo unchanged; p_u via L1 as well
+// is slower (12.04 ms: p_u rows have no reuse and evict the hot q_v lines).
+constexpr int kLcQ = 5;
 #ifndef MF_HOG_MINB
 #define MF_HOG_MINB 5
 #endif
-template <typename T, int K, int L, int D, bool ADA, bool EX, int SRC, bool GRP>
+template <typename T, int K, int L, int D, bool ADA, bool EX, int SRC, bool GRP, int LC>
 __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L > 16) ? 1 : MF_HOG_MINB)
     k_hogwild(const Rating* __restrict__ slots,
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
@@ -96,7 +102,7 @@ __global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L >
     if constexpr (SRC == 2)
       done += run_chunk_ring<T, K, L, 2, EX>(slots, lo, f, act, P, Q, st, gl, gbase, rowring);
     else
-      done += run_serial<T, K, L, D, true, ADA, EX, SRC, GRP>(slots, lo, f, act, P, Q, st, gl, gbase,
+      done += run_serial<T, K, L, D, true, ADA, EX, SRC, GRP, LC>(slots, lo, f, act, P, Q, st, gl, gbase,
                                                          0xffffffffu, ada, ring, &phase);
   }
   if (gl == 0 && done) atomicAdd(upd, (unsigned long long)done);
@@ -522,9 +528,10 @@ static Step step_of(const Launch& a) {
 }
 
 template <typename T, int K, int L, int D, bool ADA = false, bool EX = false, int SRC = 0,
-          bool GRP = false>
+          bool GRP = false, int LC = 0>
 static cudaError_t launch_hogwild_t(const HogwildLaunch& a) {
-  auto kern = k_hogwild<T, K, L, D, ADA, EX, SRC, GRP>;
+  auto kern = k_hogwild<T, K, L, D, ADA, EX, SRC, GRP, LC>;
+  if (a.out_q_l1) *a.out_q_l1 = (LC & 1);
   const int threads = 256;
   const int groups = threads / 32 * (32 / L);
   const size_t smem = SRC == 1   ? (size_t)groups * (16 + 2 * kSubBytes)
@@ -668,9 +675,13 @@ static constexpr int lanes_for(int K, int S, int LB) {
 template <typename T, int K, int LB>
 static cudaError_t hogwild_kl(const HogwildLaunch& a) {
   constexpr int S = (int)sizeof(T);
+  // q_v through L1 (R28) where a lane holds whole 16-B slices
+  constexpr bool l1ok = (K * S) / lanes_for(K, S, LB) >= 16;
   if (a.group) {                                 // column-grouped batches (R24), depth 1
     if (a.ada.GP) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, true, false, 0, true>(a);
     if (a.exact) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, true, 0, true>(a);
+    if constexpr (l1ok)
+      if (a.q_l1) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, false, 0, true, kLcQ>(a);
     return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, false, 0, true>(a);
   }
   if (a.ada.GP) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, true>(a);
@@ -679,6 +690,9 @@ static cudaError_t hogwild_kl(const HogwildLaunch& a) {
     return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, false, 1>(a);        // TMA stream
   if constexpr ((K * S) / lanes_for(K, S, LB) == 16)
     if (a.rating_stage == 2) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, false, 2>(a);
+  if constexpr (l1ok)
+    if (a.prefetch == 1 && a.q_l1)
+      return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, false, 0, false, kLcQ>(a);
   if (a.prefetch == 1) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1>(a);
   return launch_hogwild_t<T, K, lanes_for(K, S, LB), 2>(a);
 }

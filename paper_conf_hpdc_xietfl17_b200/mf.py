@@ -57,7 +57,7 @@ class Params(ctypes.Structure):
                 ("launch_blocks", ctypes.c_int32), ("exact_order", ctypes.c_int32),
                 ("rating_stage", ctypes.c_int32), ("stage_chunk", ctypes.c_int64),
                 ("group_cols", ctypes.c_int32), ("check_owners", ctypes.c_int32),
-                ("grid_cols", ctypes.c_int32)]
+                ("grid_cols", ctypes.c_int32), ("q_cache", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):
@@ -66,7 +66,8 @@ class Stats(ctypes.Structure):
                 ("sgd_launches", ctypes.c_int64), ("launches", ctypes.c_int64),
                 ("updates", ctypes.c_int64), ("bytes_per_update", ctypes.c_int64),
                 ("workers", ctypes.c_int32), ("lanes", ctypes.c_int32),
-                ("grid", ctypes.c_int32), ("block", ctypes.c_int32), ("h2d_bytes", ctypes.c_int64)]
+                ("grid", ctypes.c_int32), ("block", ctypes.c_int32), ("h2d_bytes", ctypes.c_int64),
+                ("q_l1", ctypes.c_int32)]
 
 
 _lib = None
@@ -223,7 +224,7 @@ class MF:
                  lr_rule: str = "eq9", ada_eps: float = 1e-8, launch_blocks: int = 0,
                  exact_order: bool = False, rating_stage: int = 0, stage_chunk: int = 0,
                  group_cols: bool = False, check_owners: bool = False, grid_cols: int = 0,
-                 device: int = 0, rank: int = 0, world: int = 1,
+                 q_cache: int = 0, device: int = 0, rank: int = 0, world: int = 1,
                  nccl_id: bytes | None = None, transport: int = 0, stream=None,
                  allocator: str = "torch", device_budget: int | None = None):
         L = lib()
@@ -245,6 +246,7 @@ class MF:
         p.group_cols = int(group_cols)
         p.check_owners = int(check_owners)
         p.grid_cols = int(grid_cols)
+        p.q_cache = int(q_cache)
         p.lr_rule, p.ada_eps = {"eq9": 0, "adagrad": 1}[lr_rule], ada_eps
         p.device, p.rank, p.world, p.transport = device, rank, world, transport
         self._id_buf = None

@@ -72,6 +72,10 @@ def test_create_rejects_bad_params_before_touching_a_device(L):
     assert L.mf_create(ctypes.byref(p), ctypes.byref(h)) == -1
     p.world, p.grid_a = 1, 32                                        # a / world > 16 blocks
     assert L.mf_create(ctypes.byref(p), ctypes.byref(h)) == -1
+    p.grid_a = 0
+    p.q_cache = 2                                                    # q_cache in {0, 1}
+    assert L.mf_create(ctypes.byref(p), ctypes.byref(h)) == -1
+    p.q_cache = 0
     bad = mf.Params()
     assert L.mf_create(ctypes.byref(bad), ctypes.byref(h)) == -1     # struct_size unset
     assert not h.value

@@ -131,10 +131,12 @@ def test_fullsize_fp16_hogwild_full_concurrency_20_epochs(netflix):
         assert abs(res["wavefront"] - ro) <= 0.01 * ro, (res, ro)
 
 
-@pytest.mark.parametrize("variant", [dict(group_cols=True, batch_f=1024), dict(grid_cols=1)])
+@pytest.mark.parametrize("variant", [dict(group_cols=True, batch_f=1024), dict(grid_cols=1),
+                                     dict(q_cache=1)])
 def test_fullsize_fp16_hogwild_variants_20_epochs(netflix, variant):
-    """The bench line's other Hogwild configurations -- column-grouped batches (R24) and the
-    paper's a x 1 row blocks (R27, a = 4 here) -- at full concurrency for 20 epochs: test RMSE
+    """The bench line's other Hogwild configurations -- column-grouped batches (R24), the
+    paper's a x 1 row blocks (R27, a = 4 here) and q_v loads through L2 only (q_cache = 1; the
+    default reads them through L1, R28) -- at full concurrency for 20 epochs: test RMSE
     within 1% of the oracle's own 20-epoch serial run (the golden; the variants reorder the
     updates, so the bar is the north_star Hogwild bar, not parity)."""
     gold = _golden()
