@@ -183,8 +183,8 @@ typedef struct mf_params {
                              per-instruction "cache or bypass" choice of section 4, P:L234,
                              made for the feature row with temporal reuse).  0 = auto: q_v rows
                              are read through the SM's L1 (ld.ca, write-back stores) in the
-                             Hogwild kernels with >= 16-B lanes on the Eq. 9 fast-form path
-                             (plain and column-grouped batches): a hot column is then read from
+                             Hogwild kernels on the Eq. 9 fast-form path (plain batches at
+                             prefetch 1 or 2, column-grouped batches): a hot column is then read from
                              L1 by every worker of the SM instead of by an L2 load that
                              serialises with other SMs' stores to the same line.  L1 is not
                              coherent across SMs, so a read may miss other SMs' latest store --

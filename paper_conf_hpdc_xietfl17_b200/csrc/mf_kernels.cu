@@ -675,8 +675,7 @@ static constexpr int lanes_for(int K, int S, int LB) {
 template <typename T, int K, int LB>
 static cudaError_t hogwild_kl(const HogwildLaunch& a) {
   constexpr int S = (int)sizeof(T);
-  // q_v through L1 (R28) where a lane holds whole 16-B slices
-  constexpr bool l1ok = (K * S) / lanes_for(K, S, LB) >= 16;
+  constexpr bool l1ok = true;                   // q_v through L1 (R28): plain and grouped paths
   if (a.group) {                                 // column-grouped batches (R24), depth 1
     if (a.ada.GP) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, true, false, 0, true>(a);
     if (a.exact) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, true, 0, true>(a);
@@ -694,6 +693,7 @@ static cudaError_t hogwild_kl(const HogwildLaunch& a) {
     if (a.prefetch == 1 && a.q_l1)
       return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1, false, false, 0, false, kLcQ>(a);
   if (a.prefetch == 1) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 1>(a);
+  if (a.q_l1) return launch_hogwild_t<T, K, lanes_for(K, S, LB), 2, false, false, 0, false, kLcQ>(a);
   return launch_hogwild_t<T, K, lanes_for(K, S, LB), 2>(a);
 }
 template <typename T, int K>

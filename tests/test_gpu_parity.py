@@ -283,13 +283,15 @@ def test_hogwild_one_worker_elementwise_parity_all_k(storage, k, lb, exact):
                                 dict(storage="bf16", k=64), dict(storage="fp16", k=32),
                                 dict(storage="fp16", k=128, group_cols=True, batch_f=64),
                                 dict(storage="fp16", k=128, grid_cols=1, grid_a=4),
-                                dict(storage="fp16", k=128, lane_bytes=8)])
+                                dict(storage="fp16", k=128, lane_bytes=8),
+                                dict(storage="fp16", k=32, lane_bytes=8, prefetch=2),
+                                dict(storage="fp32", k=128, prefetch=2)])
 def test_q_loads_through_l1_change_nothing_serially(kw):
     """Reading R28: q_v rows read through the SM's L1 (q_cache = 0, the default) instead of L2.
     One worker runs on one SM, whose L1 sees its own stores, so the serial run is unchanged:
     bit-identical factors to the L2-only kernel (q_cache = 1) after 2 epochs, on the ragged set,
-    for plain and column-grouped batches and the a x 1 grid; stats.q_l1 says which kernel ran
-    (8-B lanes have no L1 variant)."""
+    for plain and column-grouped batches, 8-B lanes, prefetch depth 2 and the a x 1 grid;
+    stats.q_l1 says which kernel ran."""
     R = ragged()
     out = []
     for qc in (0, 1):
@@ -300,7 +302,7 @@ def test_q_loads_through_l1_change_nothing_serially(kw):
         out.append((g.factors(), g.stats()["q_l1"]))
         g.close()
     (f0, l1), (f1, l2) = out
-    assert l2 == 0 and l1 == (0 if kw.get("lane_bytes") == 8 else 1)
+    assert l2 == 0 and l1 == 1
     for a, b in zip(f0, f1):
         assert np.array_equal(a, b)
 
