@@ -469,7 +469,11 @@ def rank_main(args, C, R=None, out=None):
                                     "DRAM carries little more than the ratings; L2 latency and the "
                                     "hot q_v rows bound it (profiles/r02_row_blocks.md)")
                                    if args.grid_cols else
-                                   ("hot q_v rows (L2 read-modify-write rate of the power-law-hot "
+                                   ("q_v through L1 (R28): the hot columns are served from L1, the "
+                                    "p_u rows stream from DRAM (~220 B per update), and the kernel is "
+                                    "bound by memory latency at ~44% issue (profiles/r02_q_l1.md)"
+                                    if args.q_cache == 0 and args.workload == "netflix" else
+                                    "hot q_v rows (L2 read-modify-write rate of the power-law-hot "
                                     "columns, profiles/r01_scaling_hot_rows.md) on Netflix; DRAM on "
                                     "Yahoo (profiles/r01g_yahoo_fp16_hogwild.md)")}
     model.close()
