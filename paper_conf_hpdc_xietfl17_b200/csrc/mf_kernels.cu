@@ -41,8 +41,12 @@ constexpr int kLcQ = 5;
 #ifndef MF_HOG_MINB
 #define MF_HOG_MINB 5
 #endif
+#ifndef MF_HOG_MINB_D2
+#define MF_HOG_MINB_D2 1
+#endif
 template <typename T, int K, int L, int D, bool ADA, bool EX, int SRC, bool GRP, int LC>
-__global__ void __launch_bounds__(256, (ADA || D > 1 || K * (int)sizeof(T) / L > 16) ? 1 : MF_HOG_MINB)
+__global__ void __launch_bounds__(256, (ADA || K * (int)sizeof(T) / L > 16) ? 1
+                                       : D > 1 ? MF_HOG_MINB_D2 : MF_HOG_MINB)
     k_hogwild(const Rating* __restrict__ slots,
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
                                                  unsigned long long* __restrict__ counter,
