@@ -482,7 +482,7 @@ def rank_main(args, C, R=None, out=None):
     e2e = None
     if not args.no_e2e and not (big and world == 1):
         e2e = run_e2e(args, R, kw, stream, C)
-    det = grp = rowb = ql2 = None
+    det = grp = rowb = ql2 = best = None
     if not args.no_deterministic and world == 1 and args.schedule == "hogwild" and not big:
         det = run_deterministic(args, R, hp, stream)
         if not args.group_cols:
@@ -491,6 +491,11 @@ def rank_main(args, C, R=None, out=None):
         if not args.grid_cols:
             rowb = run_variant(args, R, hp, stream, "hogwild on the a x 1 row-block grid (R27)",
                                grid_cols=1, q_cache=args.q_cache)
+        if not args.grid_cols and not args.group_cols:
+            best = run_variant(args, R, hp, stream,
+                               "hogwild on the a x 1 row-block grid (R27) with column-grouped "
+                               "batches (R24), f=1024", grid_cols=1, group_cols=True,
+                               batch_f=1024, q_cache=args.q_cache)
         if args.q_cache == 0:
             ql2 = run_variant(args, R, hp, stream, "hogwild, q_v loads through L2 only (q_cache = 1)",
                               q_cache=1, group_cols=bool(args.group_cols),
@@ -515,7 +520,7 @@ def rank_main(args, C, R=None, out=None):
                              "epochs": visits["epochs"], "updates_per_epoch": all_updates / args.steps,
                              "N": R.N},
             "e2e": e2e, "cpu_baseline": cpu, "deterministic": det, "grouped": grp,
-            "row_blocks": rowb, "q_l2_only": ql2,
+            "row_blocks": rowb, "row_blocks_grouped": best, "q_l2_only": ql2,
             "paper_context": "cuMF_SGD Table 5 (P:L414-415), fp16 Hogwild: Netflix 267M/s TITAN X, "
                              "613M/s P100; Hugewiki 256M/s / 710M/s (other hardware; context only)"}
     if isinstance(C, ThreadRank):

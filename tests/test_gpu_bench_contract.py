@@ -41,7 +41,7 @@ def test_bench_json_line_contract():
     cb = d["cpu_baseline"]
     assert cb["kind"] == "oracle" and cb["cores"] == 1 and cb["value"] > 0
     assert d["deterministic"]["roofline"]["frac"] > 0
-    for extra in ("grouped", "row_blocks"):
+    for extra in ("grouped", "row_blocks", "row_blocks_grouped", "q_l2_only"):
         assert d[extra]["value"] > 0 and d[extra]["exactly_once_bad_units"] == 0, extra
     assert d["row_blocks"]["grid_a"] >= 1
 

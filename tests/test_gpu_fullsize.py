@@ -132,7 +132,8 @@ def test_fullsize_fp16_hogwild_full_concurrency_20_epochs(netflix):
 
 
 @pytest.mark.parametrize("variant", [dict(group_cols=True, batch_f=1024), dict(grid_cols=1),
-                                     dict(q_cache=1)])
+                                     dict(q_cache=1),
+                                     dict(grid_cols=1, group_cols=True, batch_f=1024)])
 def test_fullsize_fp16_hogwild_variants_20_epochs(netflix, variant):
     """The bench line's other Hogwild configurations -- column-grouped batches (R24), the
     paper's a x 1 row blocks (R27, a = 4 here) and q_v loads through L2 only (q_cache = 1; the
