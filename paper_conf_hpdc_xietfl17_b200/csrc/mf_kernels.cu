@@ -44,9 +44,17 @@ constexpr int kLcQ = 5;
 #ifndef MF_HOG_MINB_D2
 #define MF_HOG_MINB_D2 1
 #endif
+// The column-grouped instantiation runs the batch-unrolled loop (mf_sgd.cuh, MF_BATCH_UNROLL) and
+// is fastest at 4 blocks (64 registers): Netflix grouped f = 1024 10.62 -> 10.12 ms, on the 4 x 1
+// row blocks 9.69 -> 9.29 ms, k = 32 7.09 -> 5.93 ms (profiles/r02_grouped_batches.md); the
+// plain rolled kernel gains nothing from 64 registers and Yahoo loses (33.3 -> 35.3 ms).
+#ifndef MF_HOG_MINB_GRP
+#define MF_HOG_MINB_GRP 4
+#endif
 template <typename T, int K, int L, int D, bool ADA, bool EX, int SRC, bool GRP, int LC>
 __global__ void __launch_bounds__(256, (ADA || K * (int)sizeof(T) / L > 16) ? 1
-                                       : D > 1 ? MF_HOG_MINB_D2 : MF_HOG_MINB)
+                                       : D > 1 ? MF_HOG_MINB_D2
+                                       : GRP   ? MF_HOG_MINB_GRP : MF_HOG_MINB)
     k_hogwild(const Rating* __restrict__ slots,
                                                  const uint32_t* __restrict__ chunks, ChunkSegs segs,
                                                  unsigned long long* __restrict__ counter,
