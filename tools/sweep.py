@@ -14,6 +14,9 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 SETS = {
     "kprec": [dict(workload="netflix", k=k, storage=s) for k in (32, 64, 128, 256)
               for s in ("fp32", "fp16", "bf16")],
+    # configs[4] with the best Hogwild configuration: a x 1 row blocks (R27) + grouped batches (R24)
+    "kprec_best": [{"workload": "netflix", "k": k, "storage": s, "grid-cols": 1, "group-cols": True,
+                    "batch-f": 1024} for k in (32, 64, 128, 256) for s in ("fp32", "fp16", "bf16")],
     # the deterministic configuration of bench.py over k and storage, and the Yahoo shape
     "det": [dict(workload="netflix", k=k, storage=s, schedule="wavefront", workers=888,
                  **{"wf-cols": 7680}, cyclic=True)
@@ -36,9 +39,12 @@ SETS = {
 }
 
 
+KEYS = ('workers', 'wf-cols', 'cyclic', 'grid-cols', 'group-cols', 'batch-f')
+
+
 def run(cfg, steps, warmup):
     cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--steps", str(steps), "--warmup",
-           str(warmup), "--no-e2e", "--no-cpu-baseline"]
+           str(warmup), "--no-e2e", "--no-cpu-baseline", "--no-deterministic"]
     for k, v in cfg.items():
         if v is True:
             cmd.append(f"--{k}")
@@ -69,7 +75,7 @@ def main():
             lines.append(f"| {cfg} | error: {d['error'][-120:]!r} |")
             continue
         c, rf = d["config"], d["roofline"]
-        lines.append(f"| {cfg.get('workload')} {('(' + ', '.join(f'{k}={v}' for k, v in cfg.items() if k in ('workers', 'wf-cols', 'cyclic')) + ')') if any(k in cfg for k in ('workers', 'wf-cols', 'cyclic')) else ''} | {c['k']} | {c['storage']} | {c['schedule']} | "
+        lines.append(f"| {cfg.get('workload')} {('(' + ', '.join(f'{k}={v}' for k, v in cfg.items() if k in KEYS) + ')') if any(k in cfg for k in KEYS) else ''} | {c['k']} | {c['storage']} | {c['schedule']} | "
                      f"{d['value']/1e9:.3f} | {d['ms_per_step']:.2f} | {rf['step_achieved']:.0f} | "
                      f"{rf['step_frac']:.3f} | {d['test_rmse']:.5f} | {d['clocks']['sm_mhz']} MHz "
                      f"{d['clocks']['reasons']} |")
