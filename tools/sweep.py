@@ -17,6 +17,15 @@ SETS = {
     # configs[4] with the best Hogwild configuration: a x 1 row blocks (R27) + grouped batches (R24)
     "kprec_best": [{"workload": "netflix", "k": k, "storage": s, "grid-cols": 1, "group-cols": True,
                     "batch-f": 1024} for k in (32, 64, 128, 256) for s in ("fp32", "fp16", "bf16")],
+    # configs[2] at HEAD: Yahoo-shaped batch-Hogwild (plain, a x 1 rows, rows + grouped) vs wavefront
+    "yahoo3": [dict(workload="yahoo", storage="fp16"), dict(workload="yahoo", storage="fp32"),
+               {"workload": "yahoo", "storage": "fp16", "grid-cols": 1},
+               {"workload": "yahoo", "storage": "fp16", "grid-cols": 1, "group-cols": True, "batch-f": 1024},
+               {"workload": "yahoo", "storage": "fp32", "grid-cols": 1},
+               dict(workload="yahoo", storage="fp32", schedule="wavefront", workers=888,
+                    **{"wf-cols": 15360}, cyclic=True),
+               dict(workload="yahoo", storage="fp16", schedule="wavefront", workers=888,
+                    **{"wf-cols": 15360}, cyclic=True)],
     # the deterministic configuration of bench.py over k and storage, and the Yahoo shape
     "det": [dict(workload="netflix", k=k, storage=s, schedule="wavefront", workers=888,
                  **{"wf-cols": 7680}, cyclic=True)
