@@ -44,6 +44,8 @@ def test_bench_json_line_contract():
     for extra in ("grouped", "row_blocks", "row_blocks_grouped", "q_l2_only"):
         assert d[extra]["value"] > 0 and d[extra]["exactly_once_bad_units"] == 0, extra
     assert d["row_blocks"]["grid_a"] >= 1
+    assert d["config"]["q_loads"].startswith("L1")          # q_cache = 0 default (R28)
+    assert d["q_l2_only"]["schedule"].startswith("hogwild, q_v loads through L2")
 
 
 def test_bench_hugewiki_one_gpu_uses_the_papers_64x1_blocks():
