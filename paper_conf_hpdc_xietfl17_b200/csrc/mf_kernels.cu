@@ -225,7 +225,21 @@ __global__ void __launch_bounds__(128) k_wavefront(const Rating* __restrict__ sl
 // Ring-staged wavefront (see run_subblock_ring): same schedule, tickets and result as
 // k_wavefront; the rows of each sub-block stream through a per-worker shared-memory ring.
 template <typename T, int K, int L, int RS, int F, bool EX>
-__global__ void __launch_bounds__(128) k_wavefront2(const Rating* __restrict__ slots,
+// Register cap of the ring wavefront.  Under __launch_bounds__(128) ptxas picked 96 registers for
+// the fp16/bf16 kernels and spilled 24 B in the per-wave epilogue; the reload then followed the
+// acquire fence's L1 invalidate (CCTL.IVALL) and went to L2 on every ticket hand-off.  With a
+// cap of 168 (126 used, no stack) on B200: fp16 39.7 -> 34.8 ms, bf16 40.7 -> 36.5 ms, fp16 k = 64
+// 31.2 -> 28.8 ms, fp32 unchanged (34.3 -> 34.2 ms) (tools/gpu/run_r02az.sh).  One warp per
+// block, 6 blocks per SM: registers do not limit the co-resident worker count.
+#ifndef MF_WF_MAXNREG
+#define MF_WF_MAXNREG 168
+#endif
+#if MF_WF_MAXNREG
+__global__ void __maxnreg__(MF_WF_MAXNREG) k_wavefront2(
+#else
+__global__ void __launch_bounds__(128) k_wavefront2(
+#endif
+                                                    const Rating* __restrict__ slots,
                                                     const uint16_t* __restrict__ dup,
                                                     const int64_t* __restrict__ sub_off,
                                                     const int32_t* __restrict__ seq,
